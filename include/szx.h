@@ -1,0 +1,197 @@
+/*
+ * szx.h -- C ABI of libszx_b200.so, the B200 (sm_100a) SZx block-wise
+ * error-bounded lossy compressor.
+ *
+ * Method: Yu et al., "Ultrafast Error-Bounded Lossy Compression for
+ * Scientific Datasets", HPDC'22 (cited as P:La-b = PAPER.md lines a-b).
+ *   - problem statement: compress N values D under |d_i - d'_i| <= e
+ *     (Formula 1); output "compressed data stream in form of
+ *     bytes" (Alg. 1 I/O);
+ *   - compress = Alg. 1 + Formulas 4/5 (P:L1024-1040,
+ *     P:L1317-1324) + zsize_array;
+ *   - decompress = Fig. 10;
+ *   - REL = value-range-relative bound (footnote 1).
+ * The byte layout of the stream is DESIGN.md section 4.
+ *
+ * Conventions (all entry points):
+ *   - Pointers named d_* are DEVICE pointers, h_* are HOST pointers.
+ *     Device buffers must be 16-byte aligned (torch allocations are).
+ *   - The caller owns every buffer; the library keeps no pointer after the
+ *     call returns.  Scratch memory is either the caller's workspace
+ *     (*_ws variants, size from *_workspace_bytes) or stream-ordered
+ *     cudaMallocAsync/cudaFreeAsync on `stream`.
+ *   - All work is enqueued on `stream` (a cudaStream_t; NULL = legacy
+ *     default stream).  Calls that return a size synchronise `stream`
+ *     before returning; *_async variants never synchronise.
+ *   - Errors are negative return values (SZX_E*); no call aborts, and a
+ *     corrupt stream is reported as SZX_ECORRUPT without out-of-bounds
+ *     accesses.  There is no CPU fallback: without a CUDA device every
+ *     compute call returns SZX_ECUDA.
+ *   - Supported GPU block sizes b: 128 and 256 (b = 128 is the paper's
+ *     choice).  Max elements per stream: 2^36.
+ */
+#ifndef SZX_B200_H
+#define SZX_B200_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum { SZX_F32 = 0, SZX_F64 = 1 } szx_dtype_t;
+/* SZX_ABS: eb is the absolute bound e.  SZX_REL: e = eb * (max - min) over
+ * the finite values of the array (footnote 1; reading R13). */
+typedef enum { SZX_ABS = 0, SZX_REL = 1 } szx_ebmode_t;
+
+enum {
+    SZX_OK = 0,
+    SZX_EINVAL = -1,   /* bad argument: dtype, mode, eb < 0 / NaN / Inf, block size, null or misaligned pointer */
+    SZX_ENOSPC = -2,   /* output (or workspace) capacity too small */
+    SZX_ECORRUPT = -3, /* stream fails validation (magic, sizes, zsize sum, payload) */
+    SZX_ECUDA = -4,    /* CUDA runtime error (or no device) */
+    SZX_ENOMEM = -5    /* stream-ordered allocation failed */
+};
+
+/* Parsed 64-byte stream header. */
+typedef struct {
+    uint32_t version;        /* 1 */
+    uint32_t dtype;          /* szx_dtype_t */
+    uint32_t eb_mode;        /* szx_ebmode_t */
+    uint32_t block_size;     /* b */
+    uint64_t n;              /* number of values */
+    double eb_user;          /* eb as passed by the caller */
+    double eb_abs;           /* absolute bound actually enforced */
+    uint64_t n_nonconst;     /* number of nonconstant blocks (nNC) */
+    uint64_t payload_bytes;  /* sum of zsize */
+    uint64_t stream_bytes;   /* total stream length implied by the header */
+} szx_header_t;
+
+/* ---------------------------------------------------------------- sizes */
+
+/* Worst-case stream bytes for n values (every block raw):
+ * 64 + al16(ceil(nB/8)) + al16(W nB) + al16(2 nB) + nB + sum ceil(len/4) + W n. */
+uint64_t szx_compress_bound(uint64_t n, szx_dtype_t dt, uint32_t block_size);
+
+/* Workspace bytes needed by szx_compress_ws / _async for n values. */
+uint64_t szx_compress_workspace_bytes(uint64_t n, szx_dtype_t dt, uint32_t block_size);
+
+/* Workspace bytes needed by szx_decompress_ws / _async to decode a stream of
+ * h->n values with block size h->block_size. */
+uint64_t szx_decompress_workspace_bytes(const szx_header_t* h);
+
+/* ------------------------------------------------------------- compress */
+
+/* Compress n values at d_in (device, dt) into d_out (device, capacity
+ * out_capacity >= szx_compress_bound).  eb: absolute bound (SZX_ABS) or
+ * value-range ratio (SZX_REL), finite and >= 0.  Allocates scratch with
+ * cudaMallocAsync on `stream`, synchronises, and returns the stream length
+ * in bytes (>= 64), or a negative SZX_E* code.  n = 0 gives a 64-byte
+ * header-only stream. */
+int64_t szx_compress(const void* d_in, szx_dtype_t dt, uint64_t n, szx_ebmode_t mode, double eb,
+                     uint32_t block_size, void* d_out, uint64_t out_capacity, void* stream);
+
+/* As szx_compress with a caller workspace d_ws of ws_bytes
+ * (>= szx_compress_workspace_bytes). */
+int64_t szx_compress_ws(const void* d_in, szx_dtype_t dt, uint64_t n, szx_ebmode_t mode, double eb,
+                        uint32_t block_size, void* d_out, uint64_t out_capacity, void* d_ws,
+                        uint64_t ws_bytes, void* stream);
+
+/* Non-blocking compress: enqueues all kernels and writes the final stream
+ * length (uint64) to d_total_bytes (device pointer).  Returns SZX_OK or a
+ * negative code for argument errors detected on the host. */
+int szx_compress_async(const void* d_in, szx_dtype_t dt, uint64_t n, szx_ebmode_t mode, double eb,
+                       uint32_t block_size, void* d_out, uint64_t out_capacity, void* d_ws,
+                       uint64_t ws_bytes, uint64_t* d_total_bytes, void* stream);
+
+/* ----------------------------------------------------------- decompress */
+
+/* Host-side parse + validation of the 64-byte header at h_bytes (host).
+ * Returns SZX_OK or SZX_ECORRUPT. */
+int szx_read_header(const void* h_bytes, uint64_t nbytes, szx_header_t* out);
+
+/* Decompress the stream (in_bytes at d_in, device) into d_out (device,
+ * out_capacity_bytes >= n * W).  Accepts a bare SZX1 stream or an SZXC
+ * shard container.  Reads the header(s) back to the host, synchronises,
+ * and returns the number of values, or a negative SZX_E* code. */
+int64_t szx_decompress(const void* d_in, uint64_t in_bytes, void* d_out,
+                       uint64_t out_capacity_bytes, void* stream);
+
+/* As szx_decompress (SZX1 only) with a caller workspace. */
+int64_t szx_decompress_ws(const void* d_in, uint64_t in_bytes, void* d_out,
+                          uint64_t out_capacity_bytes, void* d_ws, uint64_t ws_bytes, void* stream);
+
+/* Non-blocking SZX1 decode.  Of the host struct h only n, dtype and
+ * block_size are used (the expected shape, e.g. from an earlier
+ * szx_read_header); nNC and the payload size are read from the stream header
+ * in device memory and validated there, so no host round-trip is needed
+ * between a compress and a decompress.  Writes 0 (ok) or SZX_ECORRUPT
+ * (int32) to d_status (device).  Returns SZX_OK or a host-detected error. */
+int szx_decompress_async(const void* d_in, uint64_t in_bytes, const szx_header_t* h,
+                         void* d_out, uint64_t out_capacity_bytes, void* d_ws, uint64_t ws_bytes,
+                         int32_t* d_status, void* stream);
+
+/* ------------------------------------------------ end-to-end host buffers */
+
+/* Compress host data h_in into host buffer h_out (capacity out_capacity):
+ * copies in, compresses, copies the stream back.  Pinned host memory gives
+ * full PCIe/NVLink-C2C bandwidth.  Returns stream bytes or SZX_E*. */
+int64_t szx_compress_host(const void* h_in, szx_dtype_t dt, uint64_t n, szx_ebmode_t mode, double eb,
+                          uint32_t block_size, void* h_out, uint64_t out_capacity, void* stream);
+
+/* Decompress a host stream into host values.  Returns n or SZX_E*. */
+int64_t szx_decompress_host(const void* h_in, uint64_t in_bytes, void* h_out,
+                            uint64_t out_capacity_bytes, void* stream);
+
+/* ------------------------------------------------ sharded (multi-GPU) use */
+
+/* Pass 1 of a sharded compress: one read of the local shard that writes the
+ * block statistics (min/max per block of block_size values) into d_ws
+ * (ws_bytes >= szx_compress_workspace_bytes) and the shard's finite-value
+ * range as two order-preserving uint64 keys to d_range_keys[2] (device):
+ * [key(min), ~key(max)], where
+ * key(x) maps (double)x to an unsigned integer with the same total order
+ * (-0 < +0).  Combine shards with an element-wise MIN (e.g. an NCCL
+ * all-reduce MIN after flipping bit 63 to signed order).  A shard without
+ * finite values yields [UINT64_MAX, UINT64_MAX]. */
+int szx_local_range(const void* d_in, szx_dtype_t dt, uint64_t n, uint32_t block_size,
+                    uint64_t* d_range_keys, void* d_ws, uint64_t ws_bytes, void* stream);
+
+/* Pass 2 of a sharded compress: MUST follow szx_local_range on the same
+ * d_in, n, block_size, d_ws and stream.  Compresses the shard as a
+ * standalone SZX1 stream whose REL bound comes from the GLOBAL range keys
+ * d_range_keys[2] (device; szx_local_range's keys MIN-reduced over all
+ * shards); d_range_keys is ignored for SZX_ABS.
+ * Writes the stream length to d_total_bytes (device) without synchronising.
+ * The stream is byte-identical to the oracle's shard p of a P-shard SZXC
+ * container. */
+int szx_compress_shard_async(const void* d_in, szx_dtype_t dt, uint64_t n, szx_ebmode_t mode,
+                             double eb, const uint64_t* d_range_keys, uint32_t block_size,
+                             void* d_out, uint64_t out_capacity, void* d_ws, uint64_t ws_bytes,
+                             uint64_t* d_total_bytes, void* stream);
+
+/* ------------------------------------------------------------ diagnostics */
+
+/* Per-kernel device timing with CUDA events recorded on the launch stream
+ * around every kernel (off by default).  szx_timing_read fills up to cap
+ * entries of names/ms_sum/launch counts since the last reset and returns
+ * the number of kernels. */
+void szx_timing_enable(int on);
+void szx_timing_reset(void);
+int szx_timing_read(const char** names, double* ms_sum, uint64_t* launches, int cap);
+
+/* Total kernels launched by the library since load (the bench's
+ * gpu_launches count). */
+uint64_t szx_launch_count(void);
+
+/* Test hook: start the R2 escalation search r_bias bits away from
+ * Formula 4 (0 = paper behaviour; the oracle has the same hook). */
+void szx_debug_set_r_bias(int r_bias);
+
+const char* szx_strerror(int code);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* SZX_B200_H */

@@ -1,0 +1,632 @@
+// szx_api.cu -- host side of libszx_b200.so: the C ABI declared in
+// include/szx.h.  Validates arguments, lays out the stream (DESIGN.md s.4)
+// and the workspace, and enqueues the sm_100a kernels on the caller's
+// stream.  No CPU fallback: every compute path runs in the kernels below.
+#include <cuda_runtime.h>
+
+#include <atomic>
+#include <cmath>
+#include <cstring>
+#include <mutex>
+#include <vector>
+
+#include "../../include/szx.h"
+#include "szx_compress.cuh"
+#include "szx_decompress.cuh"
+
+using namespace szx;
+
+namespace {
+
+constexpr uint64_t kMaxN = 1ull << 36;
+
+std::atomic<uint64_t> g_launches{0};
+std::atomic<int> g_rbias{0};
+
+// ------------------------------------------------------------ kernel timing
+struct Timing {
+    std::mutex mu;
+    bool on = false;
+    std::vector<const char*> names;
+    std::vector<double> ms;
+    std::vector<uint64_t> cnt;
+    struct Pending { int id; cudaEvent_t a, b; };
+    std::vector<Pending> pending;
+    std::vector<cudaEvent_t> pool;
+    int id_of(const char* n) {
+        for (size_t i = 0; i < names.size(); i++) if (!strcmp(names[i], n)) return (int)i;
+        names.push_back(n); ms.push_back(0); cnt.push_back(0);
+        return (int)names.size() - 1;
+    }
+    cudaEvent_t ev() {
+        if (!pool.empty()) { cudaEvent_t e = pool.back(); pool.pop_back(); return e; }
+        cudaEvent_t e; cudaEventCreate(&e); return e;
+    }
+    void resolve() {
+        for (auto& p : pending) {
+            float t = 0;
+            cudaEventSynchronize(p.b);
+            cudaEventElapsedTime(&t, p.a, p.b);
+            ms[p.id] += t; cnt[p.id] += 1;
+            pool.push_back(p.a); pool.push_back(p.b);
+        }
+        pending.clear();
+    }
+};
+Timing& timing() { static Timing t; return t; }
+
+template <typename F>
+void launch(const char* name, cudaStream_t s, F&& f) {
+    Timing& T = timing();
+    bool on;
+    { std::lock_guard<std::mutex> g(T.mu); on = T.on; }
+    if (!on) { f(); g_launches++; return; }
+    std::lock_guard<std::mutex> g(T.mu);
+    cudaEvent_t a = T.ev(), b = T.ev();
+    cudaEventRecord(a, s);
+    f();
+    cudaEventRecord(b, s);
+    T.pending.push_back({T.id_of(name), a, b});
+    g_launches++;
+}
+
+void timing_resolve() {
+    Timing& T = timing();
+    std::lock_guard<std::mutex> g(T.mu);
+    T.resolve();
+}
+
+int sm_count() {
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    return sms > 0 ? sms : 148;
+}
+
+bool have_device() {
+    int n = 0;
+    if (cudaGetDeviceCount(&n) != cudaSuccess) { cudaGetLastError(); return false; }
+    return n > 0;
+}
+
+uint64_t* pinned_u64() {
+    static thread_local uint64_t* p = nullptr;
+    if (!p && cudaMallocHost(&p, 64) != cudaSuccess) { cudaGetLastError(); p = nullptr; }
+    return p;
+}
+
+bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; }
+int wbytes(szx_dtype_t dt) { return dt == SZX_F64 ? 8 : 4; }
+bool block_ok(uint32_t b) { return b == 128 || b == 256; }
+uint64_t cdiv(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
+
+// ------------------------------------------------------------ compress layout
+struct CLayout {
+    uint64_t nB, nW, nTB, nTC;
+    uint64_t off_keys, off_zero, zero_bytes, off_scal, off_stats, off_ncpre, total;
+};
+CLayout clayout(uint64_t n, int W, uint32_t b) {
+    CLayout L{};
+    L.nB = cdiv(n, b);
+    L.nW = cdiv(L.nB, 32);
+    L.nTB = cdiv(L.nB, 256);
+    L.nTC = L.nW;
+    L.off_keys = 0;
+    L.off_zero = 16;
+    L.zero_bytes = al16(16 + 8 * L.nTB + 8 * L.nTC);
+    L.off_scal = L.off_zero + L.zero_bytes;
+    L.off_stats = L.off_scal + 32;
+    L.off_ncpre = al16(L.off_stats + 2ull * W * L.nB);
+    L.total = al16(L.off_ncpre + 4 * L.nW + 4) + 256;
+    return L;
+}
+
+Plan make_plan(const CLayout& L, uint8_t* ws, uint64_t n, szx_dtype_t dt, szx_ebmode_t mode,
+               double eb, uint32_t b, const uint64_t* range_keys) {
+    Plan p{};
+    p.n = n; p.nB = L.nB; p.nW = L.nW;
+    p.off_mu = kHeaderBytes + al16(cdiv(L.nB, 8));
+    p.b = b; p.dtype = (uint32_t)dt; p.mode = (uint32_t)mode;
+    p.r_bias = g_rbias.load();
+    p.eb_user = eb;
+    p.range_keys = range_keys ? const_cast<uint64_t*>(range_keys) : reinterpret_cast<uint64_t*>(ws + L.off_keys);
+    p.ctr = reinterpret_cast<uint32_t*>(ws + L.off_zero);
+    p.status_b = reinterpret_cast<uint64_t*>(ws + L.off_zero + 16);
+    p.status_c = p.status_b + L.nTB;
+    p.eb_abs = reinterpret_cast<double*>(ws + L.off_scal);
+    p.nnc = reinterpret_cast<uint64_t*>(ws + L.off_scal + 8);
+    p.total = reinterpret_cast<uint64_t*>(ws + L.off_scal + 16);
+    p.stats = ws + L.off_stats;
+    p.ncpre = reinterpret_cast<uint32_t*>(ws + L.off_ncpre);
+    return p;
+}
+
+int check_compress_args(const void* d_in, szx_dtype_t dt, uint64_t n, szx_ebmode_t mode, double eb,
+                        uint32_t b, const void* d_out) {
+    if (dt != SZX_F32 && dt != SZX_F64) return SZX_EINVAL;
+    if (mode != SZX_ABS && mode != SZX_REL) return SZX_EINVAL;
+    if (!(eb >= 0.0) || !std::isfinite(eb)) return SZX_EINVAL;
+    if (!block_ok(b) || n > kMaxN) return SZX_EINVAL;
+    if (!d_out || !aligned16(d_out)) return SZX_EINVAL;
+    if (n && (!d_in || !aligned16(d_in))) return SZX_EINVAL;
+    return SZX_OK;
+}
+
+template <typename T, int VPL>
+void set_smem_attrs() {
+    static bool done = false;
+    if (done) return;
+    cudaFuncSetAttribute(k_encode<T, VPL>, cudaFuncAttributeMaxDynamicSharedMemorySize, EncodeCfg<T, VPL>::SMEM);
+    cudaFuncSetAttribute(k_decode<T, VPL>, cudaFuncAttributeMaxDynamicSharedMemorySize, DecodeCfg<T, VPL>::SMEM);
+    done = true;
+}
+
+template <typename T, int VPL>
+void enqueue_stats(const void* d_in, const Plan& p, int want_range, cudaStream_t s) {
+    constexpr int UNR = 4;
+    const uint64_t per_cta = 8 * UNR;
+    uint64_t grid = cdiv(p.nB, per_cta);
+    const uint64_t cap = (uint64_t)sm_count() * 8;
+    if (grid > cap) grid = cap;
+    if (grid == 0) grid = 1;
+    launch("k_block_stats", s, [&] {
+        k_block_stats<T, VPL, UNR><<<(unsigned)grid, 256, 0, s>>>(static_cast<const T*>(d_in), p, want_range);
+    });
+}
+
+template <typename T, int VPL>
+void enqueue_encode(const void* d_in, const Plan& p, const CLayout& L, uint8_t* out, cudaStream_t s) {
+    set_smem_attrs<T, VPL>();
+    launch("k_classify", s, [&] { k_classify<T><<<(unsigned)L.nTB, 256, 0, s>>>(p, out); });
+    using C = EncodeCfg<T, VPL>;
+    launch("k_encode", s, [&] {
+        k_encode<T, VPL><<<(unsigned)L.nTC, C::NT, C::SMEM, s>>>(static_cast<const T*>(d_in), p, out);
+    });
+}
+
+template <typename F>
+void dispatch(szx_dtype_t dt, uint32_t b, F&& f);
+
+// Enqueue the whole compression.  Returns SZX_OK or an error.
+int enqueue_compress(const void* d_in, szx_dtype_t dt, uint64_t n, szx_ebmode_t mode, double eb,
+                     uint32_t b, void* d_out, uint64_t cap, void* d_ws, uint64_t ws_bytes,
+                     uint64_t** d_total_out, cudaStream_t s) {
+    int rc = check_compress_args(d_in, dt, n, mode, eb, b, d_out);
+    if (rc) return rc;
+    if (!have_device()) return SZX_ECUDA;
+    if (cap < szx_compress_bound(n, dt, b)) return SZX_ENOSPC;
+    const int W = wbytes(dt);
+    CLayout L = clayout(n, W, b);
+    if (!d_ws || !aligned16(d_ws)) return SZX_EINVAL;
+    if (ws_bytes < L.total) return SZX_ENOSPC;
+    uint8_t* ws = static_cast<uint8_t*>(d_ws);
+    uint8_t* out = static_cast<uint8_t*>(d_out);
+    Plan p = make_plan(L, ws, n, dt, mode, eb, b, nullptr);
+    *d_total_out = p.total;
+    if (n == 0) {
+        launch("k_empty_header", s, [&] { k_empty_header<<<1, 1, 0, s>>>(out, dt, mode, b, eb, p.total); });
+        return cudaGetLastError() == cudaSuccess ? SZX_OK : SZX_ECUDA;
+    }
+    cudaMemsetAsync(ws + L.off_keys, 0xFF, 16, s);
+    cudaMemsetAsync(ws + L.off_zero, 0, L.zero_bytes, s);
+    dispatch(dt, b, [&](auto tag, auto vpl) {
+        using T = decltype(tag);
+        constexpr int V = decltype(vpl)::value;
+        enqueue_stats<T, V>(d_in, p, mode == SZX_REL, s);
+        enqueue_encode<T, V>(d_in, p, L, out, s);
+    });
+    return cudaGetLastError() == cudaSuccess ? SZX_OK : SZX_ECUDA;
+}
+
+template <int V> struct IC { static constexpr int value = V; };
+template <typename F>
+void dispatch(szx_dtype_t dt, uint32_t b, F&& f) {
+    if (dt == SZX_F32) {
+        if (b == 128) f(float(), IC<4>()); else f(float(), IC<8>());
+    } else {
+        if (b == 128) f(double(), IC<4>()); else f(double(), IC<8>());
+    }
+}
+
+int64_t finish_sync(cudaStream_t s, const uint64_t* d_val, uint64_t* out_val) {
+    uint64_t* h = pinned_u64();
+    if (!h) return SZX_ECUDA;
+    if (cudaMemcpyAsync(h, d_val, 8, cudaMemcpyDeviceToHost, s) != cudaSuccess) return SZX_ECUDA;
+    if (cudaStreamSynchronize(s) != cudaSuccess) return SZX_ECUDA;
+    timing_resolve();
+    *out_val = h[0];
+    return SZX_OK;
+}
+
+// ------------------------------------------------------------ decompress layout
+// Sized from the shape only (n, b): the number of nonconstant blocks is read
+// from the stream header on the device, so the layout covers nNC <= nB.
+struct DLayout {
+    uint64_t nB, nW, nTA, nTZmax;
+    uint64_t zero_bytes, off_ncpre, off_zpre, total;
+};
+DLayout dlayout(uint64_t n, uint32_t b) {
+    DLayout L{};
+    L.nB = cdiv(n, b);
+    L.nW = cdiv(L.nB, 32);
+    L.nTA = cdiv(L.nW, 1024);
+    L.nTZmax = cdiv(cdiv(L.nB, 32), 256);
+    L.zero_bytes = al16(16 + 16 + 8 * L.nTA + 8 * L.nTZmax);  // ctr[2], err, status_a, status_z
+    L.off_ncpre = L.zero_bytes;
+    L.off_zpre = al16(L.off_ncpre + 4 * L.nW + 4);
+    L.total = al16(L.off_zpre + 8 * (cdiv(L.nB, 32) + 1)) + 256;
+    return L;
+}
+
+int parse_header(const uint8_t* b, uint64_t nbytes, szx_header_t* h) {
+    if (!b || !h || nbytes < 64) return SZX_ECORRUPT;
+    if (memcmp(b, "SZX1", 4) != 0 || b[4] != 1 || b[7] != 0) return SZX_ECORRUPT;
+    uint64_t q[8];
+    memcpy(q, b, 64);
+    h->version = b[4];
+    h->dtype = b[5];
+    h->eb_mode = b[6];
+    h->block_size = (uint32_t)(q[1] & 0xFFFFFFFFu);
+    h->n = q[2];
+    memcpy(&h->eb_user, &q[3], 8);
+    memcpy(&h->eb_abs, &q[4], 8);
+    h->n_nonconst = q[5];
+    h->payload_bytes = q[6];
+    if (h->dtype > 1 || h->eb_mode > 1 || !block_ok(h->block_size) || h->n > kMaxN) return SZX_ECORRUPT;
+    const uint64_t W = h->dtype ? 8 : 4;
+    const uint64_t nB = cdiv(h->n, h->block_size);
+    if (h->n_nonconst > nB) return SZX_ECORRUPT;
+    const uint64_t maxz = 1 + h->block_size / 4 + W * h->block_size;
+    if (h->payload_bytes > h->n_nonconst * maxz) return SZX_ECORRUPT;
+    h->stream_bytes = kHeaderBytes + al16(cdiv(nB, 8)) + al16(W * nB) + al16(2 * h->n_nonconst) + h->payload_bytes;
+    return SZX_OK;
+}
+
+// Only h->n, h->dtype and h->block_size are used on the host; the kernels
+// read and validate the content-dependent header fields on the device.
+int enqueue_decompress(const void* d_in, uint64_t in_bytes, const szx_header_t* h, void* d_out,
+                       uint64_t cap, void* d_ws, uint64_t ws_bytes, int32_t** d_err_out, cudaStream_t s) {
+    if (!d_in || !aligned16(d_in) || !h) return SZX_EINVAL;
+    if (h->dtype > 1 || !block_ok(h->block_size) || h->n > kMaxN) return SZX_EINVAL;
+    if (in_bytes < kHeaderBytes) return SZX_ECORRUPT;
+    const uint64_t W = h->dtype ? 8 : 4;
+    if (cap < W * h->n) return SZX_ENOSPC;
+    if (h->n && (!d_out || !aligned16(d_out))) return SZX_EINVAL;
+    DLayout L = dlayout(h->n, h->block_size);
+    if (!d_ws || !aligned16(d_ws)) return SZX_EINVAL;
+    if (ws_bytes < L.total) return SZX_ENOSPC;
+    uint8_t* ws = static_cast<uint8_t*>(d_ws);
+    DPlan p{};
+    p.n = h->n; p.nB = L.nB; p.nW = L.nW;
+    p.in_bytes = in_bytes;
+    p.off_mu = kHeaderBytes + al16(cdiv(L.nB, 8));
+    p.b = h->block_size;
+    p.dtype = h->dtype;
+    p.ctr = reinterpret_cast<uint32_t*>(ws);
+    p.err = reinterpret_cast<int32_t*>(ws + 16);
+    p.status_a = reinterpret_cast<uint64_t*>(ws + 32);
+    p.status_z = p.status_a + L.nTA;
+    p.ncpre = reinterpret_cast<uint32_t*>(ws + L.off_ncpre);
+    p.zpre = reinterpret_cast<uint64_t*>(ws + L.off_zpre);
+    *d_err_out = p.err;
+    cudaMemsetAsync(ws, 0, L.zero_bytes, s);
+    if (h->n == 0) return cudaGetLastError() == cudaSuccess ? SZX_OK : SZX_ECUDA;
+    const uint8_t* in = static_cast<const uint8_t*>(d_in);
+    dispatch((szx_dtype_t)h->dtype, h->block_size, [&](auto tag, auto vpl) {
+        using T = decltype(tag);
+        constexpr int V = decltype(vpl)::value;
+        set_smem_attrs<T, V>();
+        using C = DecodeCfg<T, V>;
+        launch("k_index", s, [&] { k_index<Traits<T>::W><<<(unsigned)(L.nTA + L.nTZmax), 256, 0, s>>>(p, in); });
+        launch("k_decode", s, [&] {
+            k_decode<T, V><<<(unsigned)L.nW, C::NT, C::SMEM, s>>>(p, in, static_cast<T*>(d_out));
+        });
+    });
+    return cudaGetLastError() == cudaSuccess ? SZX_OK : SZX_ECUDA;
+}
+
+int read_device_bytes(const void* d_src, void* h_dst, uint64_t nbytes, cudaStream_t s) {
+    if (cudaMemcpyAsync(h_dst, d_src, nbytes, cudaMemcpyDeviceToHost, s) != cudaSuccess) return SZX_ECUDA;
+    if (cudaStreamSynchronize(s) != cudaSuccess) return SZX_ECUDA;
+    return SZX_OK;
+}
+
+int64_t decompress_one_sync(const void* d_in, uint64_t in_bytes, const szx_header_t* h, void* d_out,
+                            uint64_t cap, void* d_ws, uint64_t ws_bytes, cudaStream_t s) {
+    int32_t* d_err = nullptr;
+    int rc = enqueue_decompress(d_in, in_bytes, h, d_out, cap, d_ws, ws_bytes, &d_err, s);
+    if (rc) return rc;
+    int32_t err = 0;
+    if (read_device_bytes(d_err, &err, 4, s)) return SZX_ECUDA;
+    timing_resolve();
+    return err ? err : (int64_t)h->n;
+}
+
+}  // namespace
+
+// ====================================================================== C ABI
+extern "C" {
+
+uint64_t szx_compress_bound(uint64_t n, szx_dtype_t dt, uint32_t b) {
+    if (b == 0) return 0;
+    const uint64_t W = wbytes(dt);
+    const uint64_t nB = cdiv(n, b);
+    return kHeaderBytes + al16(cdiv(nB, 8)) + al16(W * nB) + al16(2 * nB) + nB + cdiv(n, 4) + nB + W * n;
+}
+
+uint64_t szx_compress_workspace_bytes(uint64_t n, szx_dtype_t dt, uint32_t b) {
+    if (!block_ok(b)) return 0;
+    return clayout(n, wbytes(dt), b).total;
+}
+
+uint64_t szx_decompress_workspace_bytes(const szx_header_t* h) {
+    if (!h || !block_ok(h->block_size)) return 0;
+    return dlayout(h->n, h->block_size).total;
+}
+
+int szx_compress_async(const void* d_in, szx_dtype_t dt, uint64_t n, szx_ebmode_t mode, double eb,
+                       uint32_t b, void* d_out, uint64_t cap, void* d_ws, uint64_t ws_bytes,
+                       uint64_t* d_total_bytes, void* stream) {
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    uint64_t* d_tot = nullptr;
+    int rc = enqueue_compress(d_in, dt, n, mode, eb, b, d_out, cap, d_ws, ws_bytes, &d_tot, s);
+    if (rc) return rc;
+    if (d_total_bytes && d_total_bytes != d_tot)
+        if (cudaMemcpyAsync(d_total_bytes, d_tot, 8, cudaMemcpyDeviceToDevice, s) != cudaSuccess) return SZX_ECUDA;
+    return SZX_OK;
+}
+
+int64_t szx_compress_ws(const void* d_in, szx_dtype_t dt, uint64_t n, szx_ebmode_t mode, double eb,
+                        uint32_t b, void* d_out, uint64_t cap, void* d_ws, uint64_t ws_bytes, void* stream) {
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    uint64_t* d_tot = nullptr;
+    int rc = enqueue_compress(d_in, dt, n, mode, eb, b, d_out, cap, d_ws, ws_bytes, &d_tot, s);
+    if (rc) return rc;
+    uint64_t total = 0;
+    if (finish_sync(s, d_tot, &total)) return SZX_ECUDA;
+    return (int64_t)total;
+}
+
+int64_t szx_compress(const void* d_in, szx_dtype_t dt, uint64_t n, szx_ebmode_t mode, double eb,
+                     uint32_t b, void* d_out, uint64_t cap, void* stream) {
+    int rc = check_compress_args(d_in, dt, n, mode, eb, b, d_out);
+    if (rc) return rc;
+    if (!have_device()) return SZX_ECUDA;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    const uint64_t wsb = szx_compress_workspace_bytes(n, dt, b);
+    void* ws = nullptr;
+    if (cudaMallocAsync(&ws, wsb, s) != cudaSuccess) { cudaGetLastError(); return SZX_ENOMEM; }
+    int64_t r = szx_compress_ws(d_in, dt, n, mode, eb, b, d_out, cap, ws, wsb, stream);
+    cudaFreeAsync(ws, s);
+    return r;
+}
+
+int szx_read_header(const void* h_bytes, uint64_t nbytes, szx_header_t* out) {
+    return parse_header(static_cast<const uint8_t*>(h_bytes), nbytes, out);
+}
+
+int szx_decompress_async(const void* d_in, uint64_t in_bytes, const szx_header_t* h, void* d_out,
+                         uint64_t cap, void* d_ws, uint64_t ws_bytes, int32_t* d_status, void* stream) {
+    if (!have_device()) return SZX_ECUDA;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    int32_t* d_err = nullptr;
+    int rc = enqueue_decompress(d_in, in_bytes, h, d_out, cap, d_ws, ws_bytes, &d_err, s);
+    if (rc) return rc;
+    if (d_status && d_status != d_err)
+        if (cudaMemcpyAsync(d_status, d_err, 4, cudaMemcpyDeviceToDevice, s) != cudaSuccess) return SZX_ECUDA;
+    return SZX_OK;
+}
+
+int64_t szx_decompress_ws(const void* d_in, uint64_t in_bytes, void* d_out, uint64_t cap, void* d_ws,
+                          uint64_t ws_bytes, void* stream) {
+    if (!d_in || in_bytes < 64) return SZX_ECORRUPT;
+    if (!have_device()) return SZX_ECUDA;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    uint8_t hb[64];
+    if (read_device_bytes(d_in, hb, 64, s)) return SZX_ECUDA;
+    szx_header_t h;
+    if (parse_header(hb, 64, &h)) return SZX_ECORRUPT;
+    return decompress_one_sync(d_in, in_bytes, &h, d_out, cap, d_ws, ws_bytes, s);
+}
+
+int64_t szx_decompress(const void* d_in, uint64_t in_bytes, void* d_out, uint64_t cap, void* stream) {
+    if (!d_in || in_bytes < 64) return SZX_ECORRUPT;
+    if (!have_device()) return SZX_ECUDA;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    uint8_t hb[64];
+    if (read_device_bytes(d_in, hb, 64, s)) return SZX_ECUDA;
+    std::vector<szx_header_t> hs;
+    std::vector<uint64_t> offs, lens, firsts;
+    if (memcmp(hb, "SZXC", 4) == 0) {
+        uint32_t P;
+        memcpy(&P, hb + 8, 4);
+        uint32_t ver;
+        memcpy(&ver, hb + 4, 4);
+        uint64_t total_n;
+        memcpy(&total_n, hb + 16, 8);
+        if (ver != 1 || P == 0 || 32 + 32ull * P > in_bytes) return SZX_ECORRUPT;
+        std::vector<uint8_t> tab(32ull * P);
+        if (read_device_bytes(static_cast<const uint8_t*>(d_in) + 32, tab.data(), tab.size(), s)) return SZX_ECUDA;
+        uint64_t expect = 0;
+        for (uint32_t i = 0; i < P; i++) {
+            uint64_t e[4];
+            memcpy(e, tab.data() + 32ull * i, 32);
+            if (e[0] != expect || e[2] % 16 || e[2] + e[3] > in_bytes || e[3] < 64) return SZX_ECORRUPT;
+            uint8_t sh[64];
+            if (read_device_bytes(static_cast<const uint8_t*>(d_in) + e[2], sh, 64, s)) return SZX_ECUDA;
+            szx_header_t h;
+            if (parse_header(sh, 64, &h) || h.n != e[1]) return SZX_ECORRUPT;
+            if (!hs.empty() && h.dtype != hs[0].dtype) return SZX_ECORRUPT;
+            hs.push_back(h); offs.push_back(e[2]); lens.push_back(e[3]); firsts.push_back(e[0]);
+            expect += e[1];
+        }
+        if (expect != total_n) return SZX_ECORRUPT;
+    } else {
+        szx_header_t h;
+        if (parse_header(hb, 64, &h)) return SZX_ECORRUPT;
+        hs.push_back(h); offs.push_back(0); lens.push_back(in_bytes); firsts.push_back(0);
+    }
+    uint64_t wsb = 0, total = 0;
+    for (auto& h : hs) { wsb = std::max<uint64_t>(wsb, szx_decompress_workspace_bytes(&h)); total += h.n; }
+    const uint64_t W = hs[0].dtype ? 8 : 4;
+    if (cap < W * total) return SZX_ENOSPC;
+    void* ws = nullptr;
+    if (cudaMallocAsync(&ws, wsb, s) != cudaSuccess) { cudaGetLastError(); return SZX_ENOMEM; }
+    int64_t r = 0;
+    for (size_t i = 0; i < hs.size() && r >= 0; i++) {
+        r = decompress_one_sync(static_cast<const uint8_t*>(d_in) + offs[i], lens[i], &hs[i],
+                                static_cast<uint8_t*>(d_out) + W * firsts[i], cap - W * firsts[i], ws, wsb, s);
+    }
+    cudaFreeAsync(ws, s);
+    return r < 0 ? r : (int64_t)total;
+}
+
+int64_t szx_compress_host(const void* h_in, szx_dtype_t dt, uint64_t n, szx_ebmode_t mode, double eb,
+                          uint32_t b, void* h_out, uint64_t cap, void* stream) {
+    if (!h_out || (n && !h_in)) return SZX_EINVAL;
+    if (!have_device()) return SZX_ECUDA;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    const uint64_t W = wbytes(dt), bound = szx_compress_bound(n, dt, b);
+    if (!block_ok(b)) return SZX_EINVAL;
+    void *d_in = nullptr, *d_out = nullptr;
+    if (cudaMallocAsync(&d_in, W * n + 16, s) != cudaSuccess) { cudaGetLastError(); return SZX_ENOMEM; }
+    if (cudaMallocAsync(&d_out, bound, s) != cudaSuccess) { cudaGetLastError(); cudaFreeAsync(d_in, s); return SZX_ENOMEM; }
+    int64_t r = SZX_ECUDA;
+    if (!n || cudaMemcpyAsync(d_in, h_in, W * n, cudaMemcpyHostToDevice, s) == cudaSuccess) {
+        r = szx_compress(d_in, dt, n, mode, eb, b, d_out, bound, stream);
+        if (r >= 0) {
+            if ((uint64_t)r > cap) r = SZX_ENOSPC;
+            else if (read_device_bytes(d_out, h_out, (uint64_t)r, s)) r = SZX_ECUDA;
+        }
+    }
+    cudaFreeAsync(d_in, s);
+    cudaFreeAsync(d_out, s);
+    return r;
+}
+
+int64_t szx_decompress_host(const void* h_in, uint64_t in_bytes, void* h_out, uint64_t cap, void* stream) {
+    if (!h_in || in_bytes < 64) return SZX_ECORRUPT;
+    if (!have_device()) return SZX_ECUDA;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    void* d_in = nullptr;
+    if (cudaMallocAsync(&d_in, in_bytes, s) != cudaSuccess) { cudaGetLastError(); return SZX_ENOMEM; }
+    int64_t r = SZX_ECUDA;
+    if (cudaMemcpyAsync(d_in, h_in, in_bytes, cudaMemcpyHostToDevice, s) == cudaSuccess) {
+        // the output size comes from the header(s); decode into a device buffer
+        uint64_t total = 0, W = 4;
+        const uint8_t* hb = static_cast<const uint8_t*>(h_in);
+        if (memcmp(hb, "SZXC", 4) == 0) {
+            memcpy(&total, hb + 16, 8);
+            if (in_bytes >= 32 + 32 + 64) {
+                uint64_t off;
+                memcpy(&off, hb + 32 + 16, 8);
+                if (off + 64 <= in_bytes) W = hb[off + 5] ? 8 : 4;
+            }
+        } else {
+            szx_header_t h;
+            if (parse_header(hb, in_bytes, &h)) { cudaFreeAsync(d_in, s); return SZX_ECORRUPT; }
+            total = h.n;
+            W = h.dtype ? 8 : 4;
+        }
+        if (W * total > cap) { cudaFreeAsync(d_in, s); return SZX_ENOSPC; }
+        void* d_out = nullptr;
+        if (cudaMallocAsync(&d_out, W * total + 16, s) != cudaSuccess) { cudaGetLastError(); cudaFreeAsync(d_in, s); return SZX_ENOMEM; }
+        r = szx_decompress(d_in, in_bytes, d_out, W * total + 16, stream);
+        if (r >= 0 && read_device_bytes(d_out, h_out, W * (uint64_t)r, s)) r = SZX_ECUDA;
+        cudaFreeAsync(d_out, s);
+    }
+    cudaFreeAsync(d_in, s);
+    return r;
+}
+
+int szx_local_range(const void* d_in, szx_dtype_t dt, uint64_t n, uint32_t b, uint64_t* d_range_keys,
+                    void* d_ws, uint64_t ws_bytes, void* stream) {
+    if (dt != SZX_F32 && dt != SZX_F64) return SZX_EINVAL;
+    if (!block_ok(b) || !d_range_keys || (n && (!d_in || !aligned16(d_in))) || n > kMaxN) return SZX_EINVAL;
+    if (!have_device()) return SZX_ECUDA;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    cudaMemsetAsync(d_range_keys, 0xFF, 16, s);
+    if (n == 0) return cudaGetLastError() == cudaSuccess ? SZX_OK : SZX_ECUDA;
+    // One pass over the shard: block statistics into the workspace (consumed
+    // by szx_compress_shard_async) and the local finite range.
+    CLayout L = clayout(n, wbytes(dt), b);
+    if (!d_ws || !aligned16(d_ws) || ws_bytes < L.total) return SZX_ENOSPC;
+    Plan p = make_plan(L, static_cast<uint8_t*>(d_ws), n, dt, SZX_REL, 0.0, b, d_range_keys);
+    dispatch(dt, b, [&](auto tag, auto vpl) {
+        using T = decltype(tag);
+        enqueue_stats<T, decltype(vpl)::value>(d_in, p, 1, s);
+    });
+    return cudaGetLastError() == cudaSuccess ? SZX_OK : SZX_ECUDA;
+}
+
+int szx_compress_shard_async(const void* d_in, szx_dtype_t dt, uint64_t n, szx_ebmode_t mode, double eb,
+                             const uint64_t* d_range_keys, uint32_t b, void* d_out, uint64_t cap,
+                             void* d_ws, uint64_t ws_bytes, uint64_t* d_total_bytes, void* stream) {
+    int rc = check_compress_args(d_in, dt, n, mode, eb, b, d_out);
+    if (rc) return rc;
+    if (mode == SZX_REL && !d_range_keys) return SZX_EINVAL;
+    if (!have_device()) return SZX_ECUDA;
+    if (cap < szx_compress_bound(n, dt, b)) return SZX_ENOSPC;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    const int W = wbytes(dt);
+    CLayout L = clayout(n, W, b);
+    if (!d_ws || !aligned16(d_ws) || ws_bytes < L.total) return SZX_ENOSPC;
+    uint8_t* ws = static_cast<uint8_t*>(d_ws);
+    uint8_t* out = static_cast<uint8_t*>(d_out);
+    Plan p = make_plan(L, ws, n, dt, mode, eb, b, mode == SZX_REL ? d_range_keys : nullptr);
+    if (n == 0) {
+        // REL with an empty shard still carries the global bound in its header
+        launch("k_empty_header", s, [&] { k_empty_header<<<1, 1, 0, s>>>(out, dt, mode, b, eb, p.total); });
+    } else {
+        // block statistics were produced by szx_local_range on this workspace
+        cudaMemsetAsync(ws + L.off_zero, 0, L.zero_bytes, s);
+        dispatch(dt, b, [&](auto tag, auto vpl) {
+            using T = decltype(tag);
+            enqueue_encode<T, decltype(vpl)::value>(d_in, p, L, out, s);
+        });
+    }
+    if (d_total_bytes && cudaMemcpyAsync(d_total_bytes, p.total, 8, cudaMemcpyDeviceToDevice, s) != cudaSuccess)
+        return SZX_ECUDA;
+    return cudaGetLastError() == cudaSuccess ? SZX_OK : SZX_ECUDA;
+}
+
+void szx_timing_enable(int on) {
+    Timing& T = timing();
+    std::lock_guard<std::mutex> g(T.mu);
+    T.on = on != 0;
+}
+void szx_timing_reset(void) {
+    Timing& T = timing();
+    std::lock_guard<std::mutex> g(T.mu);
+    T.resolve();
+    for (auto& m : T.ms) m = 0;
+    for (auto& c : T.cnt) c = 0;
+}
+int szx_timing_read(const char** names, double* ms_sum, uint64_t* launches, int cap) {
+    Timing& T = timing();
+    std::lock_guard<std::mutex> g(T.mu);
+    T.resolve();
+    int k = (int)T.names.size();
+    for (int i = 0; i < k && i < cap; i++) {
+        if (names) names[i] = T.names[i];
+        if (ms_sum) ms_sum[i] = T.ms[i];
+        if (launches) launches[i] = T.cnt[i];
+    }
+    return k;
+}
+uint64_t szx_launch_count(void) { return g_launches.load(); }
+void szx_debug_set_r_bias(int r_bias) { g_rbias.store(r_bias); }
+
+const char* szx_strerror(int code) {
+    switch (code) {
+        case SZX_OK: return "ok";
+        case SZX_EINVAL: return "invalid argument";
+        case SZX_ENOSPC: return "capacity too small";
+        case SZX_ECORRUPT: return "corrupt stream";
+        case SZX_ECUDA: return "CUDA error or no device";
+        case SZX_ENOMEM: return "allocation failed";
+        default: return "unknown error";
+    }
+}
+
+}  // extern "C"

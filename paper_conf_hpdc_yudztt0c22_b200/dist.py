@@ -1,0 +1,170 @@
+"""Multi-GPU SZx: one process per GPU, the array sharded by contiguous block ranges.
+
+The paper's compressor has no collective (blocks are independent, P:L2340-2342,
+P:L2393-2396); the only couplings of a sharded array are
+  (i)  the value-range-relative bound, which is GLOBAL (footnote 1):
+       an all-reduce MIN of two 8-byte order-preserving keys;
+  (ii) the container header: an all-gather of each shard's (n_elem, bytes) so
+       every rank knows every shard's offset in the SZXC container.
+Shard p of P owns blocks [floor(p nB / P), floor((p+1) nB / P)) (DESIGN.md s.8),
+so a container written on P GPUs decodes on one GPU and vice versa.
+
+torch.distributed (NCCL on GPUs, gloo in the CPU tests) is the plumbing; the
+codec itself is the C ABI (szx_local_range + szx_compress_shard_async).
+"""
+from __future__ import annotations
+
+import ctypes
+import struct
+
+import torch
+import torch.distributed as dist
+
+CONTAINER_HEAD = 32
+CONTAINER_ENTRY = 32
+_FLIP = -(1 << 63)  # bit 63 as int64: maps unsigned key order to signed order
+
+
+def al16(x: int) -> int:
+    return (x + 15) // 16 * 16
+
+
+def shard_blocks(nB: int, P: int, p: int) -> tuple[int, int]:
+    return nB * p // P, nB * (p + 1) // P
+
+
+def shard_elems(n: int, b: int, P: int, p: int) -> tuple[int, int]:
+    """(first element, element count) of shard p."""
+    nB = (n + b - 1) // b
+    b0, b1 = shard_blocks(nB, P, p)
+    e0, e1 = b0 * b, min(n, b1 * b)
+    return e0, max(0, e1 - e0)
+
+
+def allreduce_range_keys(keys: torch.Tensor, group=None) -> torch.Tensor:
+    """Element-wise MIN of [key(min), ~key(max)] (uint64 bit patterns held in int64) over ranks."""
+    if group is None and not (dist.is_available() and dist.is_initialized()):
+        return keys
+    if dist.get_world_size(group) == 1:
+        return keys
+    k = torch.bitwise_xor(keys, torch.full_like(keys, _FLIP))
+    dist.all_reduce(k, op=dist.ReduceOp.MIN, group=group)
+    return torch.bitwise_xor(k, torch.full_like(k, _FLIP))
+
+
+def container_layout(n_elems: list[int], nbytes: list[int]):
+    """Offsets (16-aligned) of each shard stream inside the SZXC container and its total size."""
+    P = len(n_elems)
+    pos = CONTAINER_HEAD + CONTAINER_ENTRY * P
+    offs, firsts = [], []
+    first = 0
+    for p in range(P):
+        pos = al16(pos)
+        offs.append(pos)
+        firsts.append(first)
+        pos += nbytes[p]
+        first += n_elems[p]
+    return firsts, offs, pos
+
+
+def container_header(n_elems: list[int], nbytes: list[int]) -> bytes:
+    P = len(n_elems)
+    firsts, offs, _ = container_layout(n_elems, nbytes)
+    head = bytearray(CONTAINER_HEAD + CONTAINER_ENTRY * P)
+    head[0:4] = b"SZXC"
+    struct.pack_into("<IIIQQ", head, 4, 1, P, 0, sum(n_elems), 0)
+    for p in range(P):
+        struct.pack_into("<QQQQ", head, CONTAINER_HEAD + CONTAINER_ENTRY * p, firsts[p], n_elems[p], offs[p],
+                         nbytes[p])
+    return bytes(head)
+
+
+def build_container(streams: list[torch.Tensor], n_elems: list[int]) -> torch.Tensor:
+    """Concatenate P shard streams (uint8 tensors, any device) into one SZXC container."""
+    nbytes = [int(s.numel()) for s in streams]
+    _, offs, total = container_layout(n_elems, nbytes)
+    dev = streams[0].device if streams else torch.device("cpu")
+    out = torch.zeros(total, dtype=torch.uint8, device=dev)
+    head = torch.frombuffer(bytearray(container_header(n_elems, nbytes)), dtype=torch.uint8)
+    out[:head.numel()] = head.to(dev)
+    for s, o in zip(streams, offs):
+        out[o:o + s.numel()] = s.to(dev)
+    return out
+
+
+class ShardedCompressor:
+    """Compress this rank's shard of a global array into a standalone SZX1 stream.
+
+    compress() enqueues, without host synchronisation:
+      szx_local_range (block statistics + local finite range, one read of the shard)
+      -> all-reduce MIN of the 16-byte range keys (REL only)
+      -> szx_compress_shard_async (classify + encode with the GLOBAL bound)
+      -> all-gather of (n_elem, stream bytes) so every rank knows the container offsets.
+    """
+
+    def __init__(self, n_local: int, dtype=torch.float32, block_size: int = 128, device="cuda", group=None):
+        from . import szx as _szx
+        self._szx = _szx
+        self.n, self.b, self.group = n_local, block_size, group
+        self.dtype = dtype
+        self.dt = _szx.F32 if dtype == torch.float32 else _szx.F64
+        self.cap = _szx.compress_bound(n_local, self.dt, block_size)
+        self.out = torch.empty(self.cap, dtype=torch.uint8, device=device)
+        self.ws = torch.empty(max(_szx.workspace_bytes(n_local, self.dt, block_size), 16), dtype=torch.uint8,
+                              device=device)
+        self.keys = torch.empty(2, dtype=torch.int64, device=device)
+        self.total = torch.zeros(1, dtype=torch.int64, device=device)
+        self.rec = torch.zeros(2, dtype=torch.int64, device=device)
+        ws = dist.get_world_size(group) if dist.is_available() and dist.is_initialized() else 1
+        self.world = ws
+        self.records = torch.zeros(ws, 2, dtype=torch.int64, device=device)
+
+    def compress(self, x: torch.Tensor, eb: float, mode="rel", stream=None):
+        L = self._szx.lib()
+        m = self._szx._mode_code(mode)
+        st = self._szx._stream(stream)
+        assert x.is_contiguous() and x.numel() == self.n and x.dtype == self.dtype
+        xp = x.data_ptr() if self.n else None
+        self._szx._check(L.szx_local_range(xp, self.dt, self.n, self.b, self.keys.data_ptr(), self.ws.data_ptr(),
+                                           self.ws.numel(), st), "szx_local_range")
+        if m == self._szx.REL and self.world > 1:
+            self.keys.copy_(allreduce_range_keys(self.keys, self.group))
+        self._szx._check(L.szx_compress_shard_async(xp, self.dt, self.n, m, float(eb),
+                                                    ctypes.c_void_p(self.keys.data_ptr()), self.b,
+                                                    self.out.data_ptr(), self.cap, self.ws.data_ptr(),
+                                                    self.ws.numel(), self.total.data_ptr(), st),
+                         "szx_compress_shard_async")
+        self.rec[0] = self.n
+        self.rec[1:2].copy_(self.total)
+        if self.world > 1:
+            dist.all_gather_into_tensor(self.records, self.rec, group=self.group)
+        else:
+            self.records[0].copy_(self.rec)
+
+    def stream(self) -> torch.Tensor:
+        """This rank's stream (synchronises to read its length)."""
+        return self.out[: int(self.total.item())]
+
+    def container_offsets(self):
+        """(firsts, offsets, total container bytes) from the all-gathered records (host sync)."""
+        r = self.records.cpu().tolist()
+        return container_layout([int(a) for a, _ in r], [int(bb) for _, bb in r])
+
+
+def gather_container(sc: ShardedCompressor, dst: int = 0, group=None) -> torch.Tensor | None:
+    """Collect every rank's stream on rank dst and build the SZXC container there."""
+    s = sc.stream()
+    r = sc.records.cpu().tolist()
+    n_elems = [int(a) for a, _ in r]
+    nbytes = [int(bb) for _, bb in r]
+    if sc.world == 1:
+        return build_container([s], n_elems)
+    mx = max(nbytes)
+    pad = torch.zeros(mx, dtype=torch.uint8, device=s.device)
+    pad[: s.numel()] = s
+    rank = dist.get_rank(group)
+    bufs = [torch.empty(mx, dtype=torch.uint8, device=s.device) for _ in range(sc.world)] if rank == dst else None
+    dist.gather(pad, bufs, dst=dst, group=group)
+    if rank != dst:
+        return None
+    return build_container([b[:nb] for b, nb in zip(bufs, nbytes)], n_elems)

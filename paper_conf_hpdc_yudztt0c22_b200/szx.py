@@ -1,0 +1,303 @@
+"""Thin ctypes binding of libszx_b200.so (include/szx.h).
+
+Argument marshalling only: every step of compression and decompression runs
+in the sm_100a kernels behind the C ABI.  torch provides device memory
+(``data_ptr``) and streams (``cuda_stream``).  There is no CPU fallback: if
+the library or a CUDA device is missing, every call raises.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import struct
+from dataclasses import dataclass
+
+import torch
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libszx_b200.so")
+
+F32, F64 = 0, 1
+ABS, REL = 0, 1
+_ERR = {0: "ok", -1: "EINVAL", -2: "ENOSPC", -3: "ECORRUPT", -4: "ECUDA", -5: "ENOMEM"}
+
+
+class SZxError(RuntimeError):
+    def __init__(self, code: int, what: str):
+        super().__init__(f"{what}: {_ERR.get(code, code)} ({code})")
+        self.code = code
+
+
+class _Header(ctypes.Structure):
+    _fields_ = [("version", ctypes.c_uint32), ("dtype", ctypes.c_uint32), ("eb_mode", ctypes.c_uint32),
+                ("block_size", ctypes.c_uint32), ("n", ctypes.c_uint64), ("eb_user", ctypes.c_double),
+                ("eb_abs", ctypes.c_double), ("n_nonconst", ctypes.c_uint64),
+                ("payload_bytes", ctypes.c_uint64), ("stream_bytes", ctypes.c_uint64)]
+
+
+_lib = None
+
+
+def lib() -> ctypes.CDLL:
+    """Load the in-tree CUDA library (fails loudly if it was not built)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise RuntimeError(f"{LIB_PATH} missing: run `python -c 'import __graft_entry__ as g; g.build()'`")
+    L = ctypes.CDLL(LIB_PATH)
+    u64, i64, i32, vp, dbl, u32 = (ctypes.c_uint64, ctypes.c_int64, ctypes.c_int, ctypes.c_void_p,
+                                   ctypes.c_double, ctypes.c_uint32)
+    sig = {
+        "szx_compress_bound": (u64, [u64, i32, u32]),
+        "szx_compress_workspace_bytes": (u64, [u64, i32, u32]),
+        "szx_decompress_workspace_bytes": (u64, [ctypes.POINTER(_Header)]),
+        "szx_compress": (i64, [vp, i32, u64, i32, dbl, u32, vp, u64, vp]),
+        "szx_compress_ws": (i64, [vp, i32, u64, i32, dbl, u32, vp, u64, vp, u64, vp]),
+        "szx_compress_async": (i32, [vp, i32, u64, i32, dbl, u32, vp, u64, vp, u64, vp, vp]),
+        "szx_read_header": (i32, [vp, u64, ctypes.POINTER(_Header)]),
+        "szx_decompress": (i64, [vp, u64, vp, u64, vp]),
+        "szx_decompress_ws": (i64, [vp, u64, vp, u64, vp, u64, vp]),
+        "szx_decompress_async": (i32, [vp, u64, ctypes.POINTER(_Header), vp, u64, vp, u64, vp, vp]),
+        "szx_compress_host": (i64, [vp, i32, u64, i32, dbl, u32, vp, u64, vp]),
+        "szx_decompress_host": (i64, [vp, u64, vp, u64, vp]),
+        "szx_local_range": (i32, [vp, i32, u64, u32, vp, vp, u64, vp]),
+        "szx_compress_shard_async": (i32, [vp, i32, u64, i32, dbl, vp, u32, vp, u64, vp, u64, vp, vp]),
+        "szx_timing_enable": (None, [i32]),
+        "szx_timing_reset": (None, []),
+        "szx_timing_read": (i32, [ctypes.POINTER(ctypes.c_char_p), ctypes.POINTER(dbl),
+                                  ctypes.POINTER(u64), i32]),
+        "szx_launch_count": (u64, []),
+        "szx_debug_set_r_bias": (None, [i32]),
+        "szx_strerror": (ctypes.c_char_p, [i32]),
+    }
+    for name, (res, args) in sig.items():
+        f = getattr(L, name)
+        f.restype = res
+        f.argtypes = args
+    _lib = L
+    return L
+
+
+EXPORTED = ["szx_compress_bound", "szx_compress_workspace_bytes", "szx_decompress_workspace_bytes",
+            "szx_compress", "szx_compress_ws", "szx_compress_async", "szx_read_header",
+            "szx_decompress", "szx_decompress_ws", "szx_decompress_async", "szx_compress_host",
+            "szx_decompress_host", "szx_local_range", "szx_compress_shard_async",
+            "szx_timing_enable", "szx_timing_reset", "szx_timing_read", "szx_launch_count",
+            "szx_debug_set_r_bias", "szx_strerror"]
+
+
+def _check(rc: int, what: str) -> int:
+    if rc < 0:
+        raise SZxError(int(rc), what)
+    return rc
+
+
+def _dtype_code(t: torch.Tensor) -> int:
+    if t.dtype == torch.float32:
+        return F32
+    if t.dtype == torch.float64:
+        return F64
+    raise TypeError(f"SZx compresses float32/float64 tensors, got {t.dtype}")
+
+
+def _mode_code(mode) -> int:
+    if mode in (REL, "rel", "REL"):
+        return REL
+    if mode in (ABS, "abs", "ABS"):
+        return ABS
+    raise ValueError(f"mode must be 'abs' or 'rel', got {mode!r}")
+
+
+def _stream(stream=None) -> int:
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return s.cuda_stream
+
+
+def _require_cuda(t: torch.Tensor):
+    if not t.is_cuda:
+        raise ValueError("device tensor required (use compress_host for host buffers)")
+
+
+def compress_bound(n: int, dtype_code: int, block_size: int = 128) -> int:
+    return int(lib().szx_compress_bound(n, dtype_code, block_size))
+
+
+def workspace_bytes(n: int, dtype_code: int, block_size: int = 128) -> int:
+    return int(lib().szx_compress_workspace_bytes(n, dtype_code, block_size))
+
+
+def compress(x: torch.Tensor, eb: float, mode="rel", block_size: int = 128, out: torch.Tensor | None = None,
+             workspace: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """Compress a CUDA float32/float64 tensor; returns the stream as a uint8 CUDA tensor."""
+    _require_cuda(x)
+    x = x.contiguous().view(-1)
+    dt = _dtype_code(x)
+    n = x.numel()
+    cap = compress_bound(n, dt, block_size)
+    if out is None:
+        out = torch.empty(cap, dtype=torch.uint8, device=x.device)
+    if workspace is None:
+        workspace = torch.empty(max(workspace_bytes(n, dt, block_size), 16), dtype=torch.uint8, device=x.device)
+    r = lib().szx_compress_ws(x.data_ptr() if n else None, dt, n, _mode_code(mode), float(eb), block_size,
+                              out.data_ptr(), out.numel(), workspace.data_ptr(), workspace.numel(),
+                              _stream(stream))
+    _check(r, "szx_compress")
+    return out[:r]
+
+
+@dataclass
+class Header:
+    version: int
+    dtype: int
+    eb_mode: int
+    block_size: int
+    n: int
+    eb_user: float
+    eb_abs: float
+    n_nonconst: int
+    payload_bytes: int
+    stream_bytes: int
+    _c: _Header
+
+    @property
+    def torch_dtype(self):
+        return torch.float32 if self.dtype == F32 else torch.float64
+
+
+def read_header(b: bytes) -> Header:
+    h = _Header()
+    buf = ctypes.create_string_buffer(bytes(b[:64]), 64)
+    _check(lib().szx_read_header(buf, len(b), ctypes.byref(h)), "szx_read_header")
+    return Header(h.version, h.dtype, h.eb_mode, h.block_size, h.n, h.eb_user, h.eb_abs, h.n_nonconst,
+                  h.payload_bytes, h.stream_bytes, h)
+
+
+def _container_info(stream_t: torch.Tensor):
+    head = stream_t[:64].cpu().numpy().tobytes()
+    if head[:4] == b"SZXC":
+        P = struct.unpack_from("<I", head, 8)[0]
+        n = struct.unpack_from("<Q", head, 16)[0]
+        off0 = struct.unpack_from("<Q", stream_t[32 + 16:32 + 24].cpu().numpy().tobytes())[0]
+        dt = int(stream_t[off0 + 5].item())
+        return n, dt
+    h = read_header(head)
+    return h.n, h.dtype
+
+
+def decompress(s: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """Decompress an SZX1 stream or SZXC container held in a uint8 CUDA tensor."""
+    _require_cuda(s)
+    n, dt = _container_info(s)
+    tdt = torch.float32 if dt == F32 else torch.float64
+    if out is None:
+        out = torch.empty(max(n, 1), dtype=tdt, device=s.device)
+    r = lib().szx_decompress(s.data_ptr(), s.numel(), out.data_ptr(), out.numel() * out.element_size(),
+                             _stream(stream))
+    _check(r, "szx_decompress")
+    return out[:n]
+
+
+def compress_host(x, eb: float, mode="rel", block_size: int = 128, out=None, stream=None):
+    """End-to-end compress of a HOST tensor (ideally pinned) through the C ABI's host entry point.
+    Returns a uint8 CPU tensor view of the stream."""
+    x = x.contiguous().view(-1)
+    if x.is_cuda:
+        raise ValueError("host tensor required")
+    dt = _dtype_code(x)
+    cap = compress_bound(x.numel(), dt, block_size)
+    if out is None:
+        out = torch.empty(cap, dtype=torch.uint8, pin_memory=True)
+    r = lib().szx_compress_host(x.data_ptr() if x.numel() else None, dt, x.numel(), _mode_code(mode),
+                                float(eb), block_size, out.data_ptr(), out.numel(), _stream(stream))
+    _check(r, "szx_compress_host")
+    return out[:r]
+
+
+def decompress_host(s, out=None, stream=None):
+    """End-to-end decompress of a HOST stream (uint8 CPU tensor) into a host tensor."""
+    if s.is_cuda:
+        raise ValueError("host tensor required")
+    head = s[:64].numpy().tobytes()
+    if head[:4] == b"SZXC":
+        n = struct.unpack_from("<Q", head, 16)[0]
+        off0 = struct.unpack_from("<Q", s[48:56].numpy().tobytes())[0]
+        dt = int(s[off0 + 5])
+    else:
+        h = read_header(head)
+        n, dt = h.n, h.dtype
+    tdt = torch.float32 if dt == F32 else torch.float64
+    if out is None:
+        out = torch.empty(max(n, 1), dtype=tdt, pin_memory=True)
+    r = lib().szx_decompress_host(s.data_ptr(), s.numel(), out.data_ptr(), out.numel() * out.element_size(),
+                                  _stream(stream))
+    _check(r, "szx_decompress_host")
+    return out[:n]
+
+
+class Codec:
+    """Reusable buffers for repeated compress/decompress of same-shaped arrays (bench, pipelines).
+
+    ``compress_async`` / ``decompress_async`` never synchronise: the stream length stays on
+    the device (``self.d_total``) until ``stream_bytes()`` reads it back.
+    """
+
+    def __init__(self, n: int, dtype=torch.float32, block_size: int = 128, device="cuda"):
+        self.n, self.block_size = n, block_size
+        self.dt = F32 if dtype == torch.float32 else F64
+        self.dtype = dtype
+        self.device = torch.device(device)
+        self.cap = compress_bound(n, self.dt, block_size)
+        self.out = torch.empty(self.cap, dtype=torch.uint8, device=device)
+        self.ws = torch.empty(max(workspace_bytes(n, self.dt, block_size), 16), dtype=torch.uint8, device=device)
+        self.d_total = torch.zeros(1, dtype=torch.int64, device=device)
+        self.d_status = torch.zeros(1, dtype=torch.int32, device=device)
+        self.dws = None
+
+    def compress_async(self, x: torch.Tensor, eb: float, mode="rel", stream=None):
+        assert x.is_cuda and x.numel() == self.n and x.dtype == self.dtype and x.is_contiguous()
+        rc = lib().szx_compress_async(x.data_ptr() if self.n else None, self.dt, self.n, _mode_code(mode),
+                                      float(eb), self.block_size, self.out.data_ptr(), self.cap,
+                                      self.ws.data_ptr(), self.ws.numel(), self.d_total.data_ptr(),
+                                      _stream(stream))
+        _check(rc, "szx_compress_async")
+
+    def stream_bytes(self) -> int:
+        return int(self.d_total.item())
+
+    def header(self) -> Header:
+        return read_header(self.out[:64].cpu().numpy().tobytes())
+
+    def decompress_async(self, s: torch.Tensor, h: Header, y: torch.Tensor, stream=None):
+        need = int(lib().szx_decompress_workspace_bytes(ctypes.byref(h._c)))
+        if self.dws is None or self.dws.numel() < need:
+            self.dws = torch.empty(max(need, 16), dtype=torch.uint8, device=self.device)
+        rc = lib().szx_decompress_async(s.data_ptr(), s.numel(), ctypes.byref(h._c), y.data_ptr(),
+                                        y.numel() * y.element_size(), self.dws.data_ptr(), self.dws.numel(),
+                                        self.d_status.data_ptr(), _stream(stream))
+        _check(rc, "szx_decompress_async")
+
+
+def timing_enable(on: bool = True):
+    lib().szx_timing_enable(1 if on else 0)
+
+
+def timing_reset():
+    lib().szx_timing_reset()
+
+
+def timing_read() -> dict:
+    names = (ctypes.c_char_p * 32)()
+    ms = (ctypes.c_double * 32)()
+    cnt = (ctypes.c_uint64 * 32)()
+    k = lib().szx_timing_read(names, ms, cnt, 32)
+    return {names[i].decode(): (ms[i], int(cnt[i])) for i in range(min(k, 32))}
+
+
+def launch_count() -> int:
+    return int(lib().szx_launch_count())
+
+
+def set_r_bias(r: int):
+    """Test hook (see szx_debug_set_r_bias)."""
+    lib().szx_debug_set_r_bias(int(r))

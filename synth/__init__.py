@@ -79,9 +79,10 @@ def hurricane_like(field: int = 0, shape=(100, 500, 500), device="cpu") -> torch
 
 
 # ---- config 3: NYX 512^3 ----------------------------------------------
-def nyx_like(field: int = 0, n: int = 512, device="cpu") -> torch.Tensor:
-    """(0) baryon-density-like exp(2.5 g); (1) velocity-like g; (2) temperature-like exp(0.7 g)."""
-    g = grf((n, n, n), 4.0, 1000 + 10 * 3 + field, device)
+def nyx_like(field: int = 0, n: int = 512, device="cpu", seed_offset: int = 0) -> torch.Tensor:
+    """(0) baryon-density-like exp(2.5 g); (1) velocity-like g; (2) temperature-like exp(0.7 g).
+    seed_offset selects another realisation (one per rank in weak-scaling runs)."""
+    g = grf((n, n, n), 4.0, 1000 + 10 * 3 + field + 100000 * seed_offset, device)
     if field == 0:
         return torch.exp(2.5 * g).contiguous()
     if field == 1:
