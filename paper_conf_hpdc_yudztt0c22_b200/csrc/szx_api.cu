@@ -103,21 +103,22 @@ uint64_t cdiv(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
 // ------------------------------------------------------------ compress layout
 struct CLayout {
     uint64_t nB, nW, nTB, nTC;
-    uint64_t off_keys, off_zero, zero_bytes, off_scal, off_stats, off_ncpre, total;
+    uint64_t off_keys, off_zero, zero_bytes, off_scal, off_stats, off_nclist, off_nckeys, total;
 };
 CLayout clayout(uint64_t n, int W, uint32_t b) {
     CLayout L{};
     L.nB = cdiv(n, b);
     L.nW = cdiv(L.nB, 32);
-    L.nTB = cdiv(L.nB, 256);
-    L.nTC = L.nW;
+    L.nTB = cdiv(L.nB, kClassifyBlocks);
+    L.nTC = cdiv(L.nB, 16);  // encode tiles hold >= 16 nonconstant blocks
     L.off_keys = 0;
     L.off_zero = 16;
     L.zero_bytes = al16(16 + 8 * L.nTB + 8 * L.nTC);
     L.off_scal = L.off_zero + L.zero_bytes;
     L.off_stats = L.off_scal + 32;
-    L.off_ncpre = al16(L.off_stats + 2ull * W * L.nB);
-    L.total = al16(L.off_ncpre + 4 * L.nW + 4) + 256;
+    L.off_nclist = al16(L.off_stats + 2ull * W * L.nB);
+    L.off_nckeys = al16(L.off_nclist + 4 * L.nB + 4);
+    L.total = al16(L.off_nckeys + 2ull * W * L.nB + 16) + 256;  // +16: TMA reads whole 16 B chunks
     return L;
 }
 
@@ -137,7 +138,8 @@ Plan make_plan(const CLayout& L, uint8_t* ws, uint64_t n, szx_dtype_t dt, szx_eb
     p.nnc = reinterpret_cast<uint64_t*>(ws + L.off_scal + 8);
     p.total = reinterpret_cast<uint64_t*>(ws + L.off_scal + 16);
     p.stats = ws + L.off_stats;
-    p.ncpre = reinterpret_cast<uint32_t*>(ws + L.off_ncpre);
+    p.nclist = reinterpret_cast<uint32_t*>(ws + L.off_nclist);
+    p.nckeys = ws + L.off_nckeys;
     return p;
 }
 
@@ -161,12 +163,18 @@ void set_smem_attrs() {
     done = true;
 }
 
+// grid-stride streaming pass: enough CTAs to fill every SM, each warp keeping
+// UNR blocks (128 bytes per lane) of loads in flight
 template <typename T, int VPL>
 void enqueue_stats(const void* d_in, const Plan& p, int want_range, cudaStream_t s) {
-    constexpr int UNR = 4;
-    const uint64_t per_cta = 8 * UNR;
-    uint64_t grid = cdiv(p.nB, per_cta);
-    const uint64_t cap = (uint64_t)sm_count() * 8;
+    constexpr int UNR = 128 / (VPL * (int)sizeof(T)) > 0 ? 128 / (VPL * (int)sizeof(T)) : 1;
+    static int occ = 0;
+    if (!occ) {
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_block_stats<T, VPL, UNR>, 256, 0);
+        if (occ <= 0) occ = 4;
+    }
+    uint64_t grid = cdiv(p.nB, 8 * UNR);
+    const uint64_t cap = (uint64_t)sm_count() * occ;
     if (grid > cap) grid = cap;
     if (grid == 0) grid = 1;
     launch("k_block_stats", s, [&] {
@@ -174,13 +182,24 @@ void enqueue_stats(const void* d_in, const Plan& p, int want_range, cudaStream_t
     });
 }
 
+// classify (ticketed look-back tiles) then the persistent encoder: one wave of
+// CTAs, all co-resident (required by the look-back across round-robin tiles)
 template <typename T, int VPL>
 void enqueue_encode(const void* d_in, const Plan& p, const CLayout& L, uint8_t* out, cudaStream_t s) {
     set_smem_attrs<T, VPL>();
     launch("k_classify", s, [&] { k_classify<T><<<(unsigned)L.nTB, 256, 0, s>>>(p, out); });
     using C = EncodeCfg<T, VPL>;
+    static int occ = 0;
+    if (!occ) {
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_encode<T, VPL>, C::NT, C::SMEM);
+        if (occ <= 0) occ = 1;
+    }
+    uint64_t grid = cdiv(L.nB, C::TB);
+    const uint64_t cap = (uint64_t)sm_count() * occ;
+    if (grid > cap) grid = cap;
+    if (grid == 0) grid = 1;
     launch("k_encode", s, [&] {
-        k_encode<T, VPL><<<(unsigned)L.nTC, C::NT, C::SMEM, s>>>(static_cast<const T*>(d_in), p, out);
+        k_encode<T, VPL><<<(unsigned)grid, C::NT, C::SMEM, s>>>(static_cast<const T*>(d_in), p, out);
     });
 }
 
@@ -204,7 +223,7 @@ int enqueue_compress(const void* d_in, szx_dtype_t dt, uint64_t n, szx_ebmode_t 
     Plan p = make_plan(L, ws, n, dt, mode, eb, b, nullptr);
     *d_total_out = p.total;
     if (n == 0) {
-        launch("k_empty_header", s, [&] { k_empty_header<<<1, 1, 0, s>>>(out, dt, mode, b, eb, p.total); });
+        launch("k_empty_header", s, [&] { k_empty_header<<<1, 1, 0, s>>>(out, dt, mode, b, eb, nullptr, p.total); });
         return cudaGetLastError() == cudaSuccess ? SZX_OK : SZX_ECUDA;
     }
     cudaMemsetAsync(ws + L.off_keys, 0xFF, 16, s);
@@ -242,19 +261,18 @@ int64_t finish_sync(cudaStream_t s, const uint64_t* d_val, uint64_t* out_val) {
 // Sized from the shape only (n, b): the number of nonconstant blocks is read
 // from the stream header on the device, so the layout covers nNC <= nB.
 struct DLayout {
-    uint64_t nB, nW, nTA, nTZmax;
-    uint64_t zero_bytes, off_ncpre, off_zpre, total;
+    uint64_t nB, nW, nTI;
+    uint64_t zero_bytes, off_ncpre, off_tbase, total;
 };
 DLayout dlayout(uint64_t n, uint32_t b) {
     DLayout L{};
     L.nB = cdiv(n, b);
     L.nW = cdiv(L.nB, 32);
-    L.nTA = cdiv(L.nW, 1024);
-    L.nTZmax = cdiv(cdiv(L.nB, 32), 256);
-    L.zero_bytes = al16(16 + 16 + 8 * L.nTA + 8 * L.nTZmax);  // ctr[2], err, status_a, status_z
+    L.nTI = cdiv(L.nW, kIndexTiles);
+    L.zero_bytes = al16(16 + 16 + 16 * L.nTI);  // ctr[2], err, status_a, status_z
     L.off_ncpre = L.zero_bytes;
-    L.off_zpre = al16(L.off_ncpre + 4 * L.nW + 4);
-    L.total = al16(L.off_zpre + 8 * (cdiv(L.nB, 32) + 1)) + 256;
+    L.off_tbase = al16(L.off_ncpre + 4 * L.nW + 4);
+    L.total = al16(L.off_tbase + 8 * (L.nW + 1)) + 256;
     return L;
 }
 
@@ -305,9 +323,9 @@ int enqueue_decompress(const void* d_in, uint64_t in_bytes, const szx_header_t* 
     p.ctr = reinterpret_cast<uint32_t*>(ws);
     p.err = reinterpret_cast<int32_t*>(ws + 16);
     p.status_a = reinterpret_cast<uint64_t*>(ws + 32);
-    p.status_z = p.status_a + L.nTA;
+    p.status_z = p.status_a + L.nTI;
     p.ncpre = reinterpret_cast<uint32_t*>(ws + L.off_ncpre);
-    p.zpre = reinterpret_cast<uint64_t*>(ws + L.off_zpre);
+    p.tbase = reinterpret_cast<uint64_t*>(ws + L.off_tbase);
     *d_err_out = p.err;
     cudaMemsetAsync(ws, 0, L.zero_bytes, s);
     if (h->n == 0) return cudaGetLastError() == cudaSuccess ? SZX_OK : SZX_ECUDA;
@@ -317,9 +335,17 @@ int enqueue_decompress(const void* d_in, uint64_t in_bytes, const szx_header_t* 
         constexpr int V = decltype(vpl)::value;
         set_smem_attrs<T, V>();
         using C = DecodeCfg<T, V>;
-        launch("k_index", s, [&] { k_index<Traits<T>::W><<<(unsigned)(L.nTA + L.nTZmax), 256, 0, s>>>(p, in); });
+        launch("k_index", s, [&] { k_index<Traits<T>::W><<<(unsigned)L.nTI, 256, 0, s>>>(p, in); });
+        static int occ = 0;
+        if (!occ) {
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_decode<T, V>, C::NT, C::SMEM);
+            if (occ <= 0) occ = 1;
+        }
+        uint64_t grid = L.nW;
+        const uint64_t cap = (uint64_t)sm_count() * occ;
+        if (grid > cap) grid = cap;
         launch("k_decode", s, [&] {
-            k_decode<T, V><<<(unsigned)L.nW, C::NT, C::SMEM, s>>>(p, in, static_cast<T*>(d_out));
+            k_decode<T, V><<<(unsigned)grid, C::NT, C::SMEM, s>>>(p, in, static_cast<T*>(d_out));
         });
     });
     return cudaGetLastError() == cudaSuccess ? SZX_OK : SZX_ECUDA;
@@ -576,7 +602,7 @@ int szx_compress_shard_async(const void* d_in, szx_dtype_t dt, uint64_t n, szx_e
     Plan p = make_plan(L, ws, n, dt, mode, eb, b, mode == SZX_REL ? d_range_keys : nullptr);
     if (n == 0) {
         // REL with an empty shard still carries the global bound in its header
-        launch("k_empty_header", s, [&] { k_empty_header<<<1, 1, 0, s>>>(out, dt, mode, b, eb, p.total); });
+        launch("k_empty_header", s, [&] { k_empty_header<<<1, 1, 0, s>>>(out, dt, mode, b, eb, mode == SZX_REL ? d_range_keys : nullptr, p.total); });
     } else {
         // block statistics were produced by szx_local_range on this workspace
         cudaMemsetAsync(ws + L.off_zero, 0, L.zero_bytes, s);

@@ -1,20 +1,24 @@
 // szx_decompress.cuh -- SZx decompression kernels for sm_100a.
 //
-//   k_index   (K5a) two single-pass decoupled-look-back scans in one launch:
-//             (a) nonconstant index per bitmap word = prefix of popcounts,
-//             (b) payload byte offset per group of 32 nonconstant blocks =
-//                 prefix of zsize (the paper's "prefix-sum step to compute
-//                 the starting location of each block").
-//             Both totals are validated against the header (nNC, payload).
-//   k_decode  (K5)  a CTA per tile of 32 blocks: stage the tile's payload
-//             bytes in shared memory with 16-byte loads, then a warp per
-//             block rebuilds each value with the five steps of Fig. 10
-//             (P:L2321-2336).  The leading-byte dependence chains
-//             (Challenge 2) are resolved by a warp scan of
+//   k_index   (K5a) the paper's "prefix-sum step to compute the starting
+//             location of each block", as two chained
+//             single-pass decoupled look-back scans per CTA of 256 tiles
+//             (tile = 32 blocks = one bitmap word):
+//               (a) nonconstant index of each tile = prefix of popcounts,
+//               (b) payload byte offset of each tile = prefix of its zsize
+//                   sums (the CTA's zsize range is staged in shared memory).
+//             Totals are validated against the header (nNC, payload size).
+//   k_decode  (K5)  persistent and warp-specialised: a producer warp reads a
+//             tile's metadata and issues ONE TMA bulk copy of the tile's
+//             contiguous payload (plus one for its 32 mu values) into a
+//             shared-memory ring; 8 consumer warps rebuild the values with
+//             the five steps of Fig. 10 and write them with
+//             16-byte stores.  The leading-byte dependence chains
+//             (Challenge 2) are resolved with a warp scan of
 //             byte-mask transfer functions instead of the paper's log-step
-//             index propagation: lane l's values map an
-//             incoming previous word c to (c & M_l) | D_l, and composing
-//             those maps is associative.
+//             index propagation: a lane's values map an
+//             incoming previous word c to (c & M) | D, and composing such
+//             maps is associative.
 #pragma once
 
 #include "szx_device.cuh"
@@ -30,15 +34,15 @@ struct DPlan {
     uint32_t* ctr;             // [2] tickets, init 0
     uint64_t* status_a;        // init 0
     uint64_t* status_z;        // init 0
-    uint32_t* ncpre;           // [nW]
-    uint64_t* zpre;            // [ceil(nB/32) + 1]
+    uint32_t* ncpre;           // [nW]      nonconstant index of each tile's first block
+    uint64_t* tbase;           // [nW + 1]  payload offset of each tile (tbase[nW] = total)
     int32_t* err;              // 0 ok, else SZX_ECORRUPT
 };
 
 // Stream facts read from the 64-byte header in device memory, validated
 // against the caller's shape.
 struct DHdr {
-    uint64_t nnc, payload_bytes, off_zs, off_pl, ngroups;
+    uint64_t nnc, payload_bytes, off_zs, off_pl;
     bool ok;
 };
 template <int W>
@@ -55,7 +59,6 @@ __device__ inline DHdr read_dheader(const uint8_t* in, const DPlan& p) {
     d.off_zs = p.off_mu + al16((uint64_t)W * p.nB);
     d.off_pl = d.off_zs + al16(2 * d.nnc);
     d.ok = d.ok && d.off_pl + d.payload_bytes <= p.in_bytes;
-    d.ngroups = (d.nnc + 31) / 32;
     return d;
 }
 
@@ -70,6 +73,7 @@ __device__ inline uint64_t cta_scan256(uint64_t v, uint64_t* agg, uint64_t* s_w 
         uint64_t t = __shfl_up_sync(0xffffffffu, incl, o);
         if (lane >= o) incl += t;
     }
+    __syncthreads();  // s_w may still be read by a previous scan
     if (lane == 31) s_w[warp] = incl;
     __syncthreads();
     uint64_t wpre = 0, tot = 0;
@@ -83,9 +87,12 @@ __device__ inline uint64_t cta_scan256(uint64_t v, uint64_t* agg, uint64_t* s_w 
     return wpre + incl - v;
 }
 
+constexpr int kIndexTiles = 256;  // tiles (bitmap words) per k_index CTA
+
 template <int W>
 __global__ void __launch_bounds__(256) k_index(DPlan p, const uint8_t* __restrict__ in) {
-    __shared__ uint64_t s_tile, s_excl, s_w[8];
+    __shared__ uint64_t s_tile, s_ga, s_gb, s_w[8];
+    __shared__ uint16_t s_zs[kIndexTiles * 32];
     const DHdr hd = read_dheader<W>(in, p);
     if (!hd.ok) {
         if (blockIdx.x == 0 && threadIdx.x == 0) set_corrupt(p.err);
@@ -94,86 +101,63 @@ __global__ void __launch_bounds__(256) k_index(DPlan p, const uint8_t* __restric
     if (threadIdx.x == 0) s_tile = atomicAdd(&p.ctr[0], 1u);
     __syncthreads();
     const uint64_t t = s_tile;
-    const uint64_t nTA = (p.nW + 1023) / 1024;
-    const uint64_t nTZ = (hd.ngroups + 255) / 256;
-    if (t >= nTA + nTZ) return;  // grid is sized for the largest possible nNC
-    const int warp = threadIdx.x >> 5;
-    if (t < nTA) {
-        // (a) popcount prefix over bitmap words, 4 words per thread
-        const uint32_t* bm = reinterpret_cast<const uint32_t*>(in + kHeaderBytes);
-        const uint64_t w0 = t * 1024 + threadIdx.x * 4;
-        uint32_t c[4];
-        uint64_t sum = 0;
-#pragma unroll
-        for (int q = 0; q < 4; q++) {
-            const uint64_t w = w0 + q;
-            uint32_t word = w < p.nW ? bm[w] : 0u;
-            if (w == p.nW - 1 && (p.nB & 31)) word &= (1u << (p.nB & 31)) - 1u;  // ignore padding bits
-            c[q] = __popc(word);
-            sum += c[q];
-        }
-        uint64_t agg;
-        uint64_t ex = cta_scan256(sum, &agg, s_w);
-        if (warp == 0) {
-            const uint64_t e = lookback_exclusive(p.status_a, t, agg);
-            if ((threadIdx.x & 31) == 0) {
-                s_excl = e;
-                if (t == nTA - 1 && e + agg != hd.nnc) set_corrupt(p.err);
-            }
-        }
-        __syncthreads();
-        ex += s_excl;
-#pragma unroll
-        for (int q = 0; q < 4; q++) {
-            if (w0 + q < p.nW) p.ncpre[w0 + q] = (uint32_t)ex;
-            ex += c[q];
-        }
-    } else {
-        // (b) zsize sums per group of 32 entries
-        const uint64_t tz = t - nTA;
-        const uint16_t* zs = reinterpret_cast<const uint16_t*>(in + hd.off_zs);
-        const uint64_t g = tz * 256 + threadIdx.x;
-        uint64_t sum = 0;
-        if (g < hd.ngroups) {
-            const uint64_t e0 = g * 32;
-            if (e0 + 32 <= hd.nnc) {
-                const uint4* q4 = reinterpret_cast<const uint4*>(zs + e0);
-#pragma unroll
-                for (int q = 0; q < 4; q++) {
-                    const uint4 v = q4[q];
-                    const uint32_t a[4] = {v.x, v.y, v.z, v.w};
-#pragma unroll
-                    for (int r = 0; r < 4; r++) sum += (a[r] & 0xFFFFu) + (a[r] >> 16);
-                }
-            } else {
-                for (uint64_t e = e0; e < hd.nnc; e++) sum += zs[e];
-            }
-        }
-        uint64_t agg;
-        uint64_t ex = cta_scan256(sum, &agg, s_w);
-        if (warp == 0) {
-            const uint64_t e = lookback_exclusive(p.status_z, tz, agg);
-            if ((threadIdx.x & 31) == 0) {
-                s_excl = e;
-                if (tz == nTZ - 1) {
-                    p.zpre[hd.ngroups] = e + agg;
-                    if (e + agg != hd.payload_bytes) set_corrupt(p.err);
-                }
-            }
-        }
-        __syncthreads();
-        if (g < hd.ngroups) p.zpre[g] = ex + s_excl;
+    const uint64_t ntiles = (p.nW + kIndexTiles - 1) / kIndexTiles;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint64_t w = t * kIndexTiles + threadIdx.x;
+    // (a) nonconstant index of each tile
+    uint32_t word = w < p.nW ? reinterpret_cast<const uint32_t*>(in + kHeaderBytes)[w] : 0u;
+    if (w == p.nW - 1 && (p.nB & 31)) word &= (1u << (p.nB & 31)) - 1u;  // ignore padding bits
+    const uint32_t cnt = __popc(word);
+    uint64_t aggA;
+    const uint64_t exA = cta_scan256(cnt, &aggA, s_w);
+    if (warp == 0) {
+        const uint64_t e = lookback_exclusive(p.status_a, t, aggA);
+        if (lane == 0) s_ga = e;
     }
+    __syncthreads();
+    const uint64_t GA = s_ga;
+    const uint64_t ncb = GA + exA;
+    if (w < p.nW) p.ncpre[w] = (uint32_t)ncb;
+    bool ok = GA + aggA <= hd.nnc;
+    // (b) stage this CTA's zsize entries [GA, GA + aggA) and sum per tile
+    const uint16_t* zs = reinterpret_cast<const uint16_t*>(in + hd.off_zs);
+    const uint64_t nz = ok ? aggA : 0;
+    for (uint64_t j = threadIdx.x; j < nz; j += 256) s_zs[j] = zs[GA + j];
+    __syncthreads();
+    uint64_t sum = 0;
+    if (ok)
+        for (uint32_t j = 0; j < cnt; j++) sum += s_zs[exA + j];
+    uint64_t aggB;
+    const uint64_t exB = cta_scan256(sum, &aggB, s_w);
+    if (warp == 0) {
+        const uint64_t e = lookback_exclusive(p.status_z, t, aggB);
+        if (lane == 0) {
+            s_gb = e;
+            if (t == ntiles - 1) {
+                p.tbase[p.nW] = e + aggB;
+                if (GA + aggA != hd.nnc || e + aggB != hd.payload_bytes) set_corrupt(p.err);
+            }
+        }
+    }
+    if (!__syncthreads_and(ok ? 1 : 0) && threadIdx.x == 0) set_corrupt(p.err);
+    if (w < p.nW) p.tbase[w] = s_gb + exB;
 }
 
 template <typename T, int VPL>
 struct DecodeCfg {
+    static constexpr int W = Traits<T>::W;
     static constexpr int B = 32 * VPL;
-    static constexpr int BPW = VPL == 4 ? 4 : 2;
-    static constexpr int NWARP = kTileBlocks / BPW;
-    static constexpr int NT = NWARP * 32;
-    static constexpr int MAXZ = 1 + B / 4 + Traits<T>::W * B;
-    static constexpr int SMEM = 16 + kTileBlocks * MAXZ + 16;
+    static constexpr int TB = kTileBlocks;                 // blocks per tile (one bitmap word)
+    static constexpr int NWARP = 8;                        // consumer warps
+    static constexpr int BPW = TB / NWARP;
+    static constexpr int NT = (NWARP + 1) * 32;            // + producer warp
+    static constexpr int MAXZ = 1 + B / 4 + W * B;
+    static constexpr int PAY = (TB * MAXZ + 32 + 15) / 16 * 16;  // + up to 15 lead / trail bytes
+    static constexpr int MUB = TB * W;
+    static constexpr int STAGE = PAY + MUB;
+    static constexpr int STAGES = (W == 4 && VPL == 4) ? 3 : 2;
+    static constexpr int SMEM = STAGES * STAGE;
+    static constexpr int MINB = (W == 4 && VPL == 4) ? 3 : 2;
 };
 
 template <typename T, int VPL>
@@ -223,17 +207,24 @@ __device__ inline bool decode_block(const uint8_t* src, uint32_t z, int len, T m
     const uint32_t incl = warp_incl_scan(m);
     const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
     if (1u + (uint32_t)ncode + total != z) return false;
-    // (3) mid-bytes -> own bytes, and the byte-mask transfer function of this lane
-    const uint8_t* mb = src + 1 + ncode + (incl - m);
+    // (3) mid-bytes -> own bytes, and the byte-mask transfer function of this lane.
+    // The lane's run of mid-bytes is read as aligned words and realigned with
+    // funnel shifts; value i takes the next m_i bytes of the run.
+    constexpr int NW = VPL * W / 4;
+    uint32_t run[NW];
+    run_load<NW>(src + 1 + ncode + (incl - m), run);
     U own[VPL];
     U M = ~U(0), D = 0;  // lane map: c -> (c & M) | D
-    int pos = 0;
 #pragma unroll
     for (int i = 0; i < VPL; i++) {
         own[i] = 0;
         if (i < cnt) {
             const int L = (leads >> (2 * i)) & 3;
-            for (int j = W - req; j < W - L; j++) own[i] |= (U)mb[pos++] << (8 * j);
+            const int mi = req > L ? req - L : 0;
+            U bytes = W == 4 ? (U)run[0] : ((U)run[0] | ((U)run[1] << 16 << 16));
+            bytes &= mi >= W ? ~U(0) : ((U(1) << (8 * mi)) - U(1));
+            own[i] = bytes << (8 * (W - req));
+            run_shr<NW>(run, mi);
             const int copy = L < req ? L : req;
             // bytes copied from the previous value: the top `copy` bytes (step 2)
             const U cm = copy == 0 ? U(0) : (~U(0) << (8 * (W - copy)));
@@ -270,93 +261,144 @@ __device__ inline bool decode_block(const uint8_t* src, uint32_t z, int len, T m
 }
 
 template <typename T, int VPL>
-__global__ void __launch_bounds__(DecodeCfg<T, VPL>::NT)
+__global__ void __launch_bounds__(DecodeCfg<T, VPL>::NT, DecodeCfg<T, VPL>::MINB)
     k_decode(DPlan p, const uint8_t* __restrict__ in, T* __restrict__ y) {
     using TR = Traits<T>;
     using U = typename TR::U;
     using C = DecodeCfg<T, VPL>;
-    extern __shared__ __align__(16) uint8_t stg[];
-    __shared__ uint32_t s_off[kTileBlocks], s_z[kTileBlocks];
-    __shared__ uint64_t s_base;
-    __shared__ int s_ok;
+    extern __shared__ __align__(128) uint8_t smem[];
+    __shared__ __align__(8) uint64_t full_bar[C::STAGES], empty_bar[C::STAGES];
+    __shared__ __align__(16) uint16_t s_zw[C::STAGES][C::TB + 16];  // zsize window (TMA)
+    __shared__ uint32_t s_word[C::STAGES], s_sb[C::STAGES], s_zo[C::STAGES], s_ok[C::STAGES];
+    __shared__ uint64_t s_T[C::STAGES];
+
     const DHdr hd = read_dheader<TR::W>(in, p);
     if (!hd.ok) return;  // k_index has flagged it
-    const uint64_t tile = blockIdx.x;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    uint32_t word = reinterpret_cast<const uint32_t*>(in + kHeaderBytes)[tile];
-    if (tile == p.nW - 1 && (p.nB & 31)) word &= (1u << (p.nB & 31)) - 1u;
-    const uint32_t cnt = __popc(word);
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < C::STAGES; s++) {
+            mbar_init(&full_bar[s], 1);
+            mbar_init(&empty_bar[s], C::NWARP);
+        }
+        fence_mbar_init();
+    }
+    __syncthreads();
+    const uint64_t G = gridDim.x;
 
-    if (warp == 0) {
-        const uint64_t ncb = p.ncpre[tile];
-        const uint16_t* zs = reinterpret_cast<const uint16_t*>(in + hd.off_zs);
-        bool ok = ncb + cnt <= hd.nnc;
-        uint64_t base = 0;
-        uint32_t zl = 0;
-        if (ok && cnt) {
-            const uint64_t g0 = ncb & ~uint64_t(31);
-            const uint64_t e = g0 + lane;
-            const uint32_t part = warp_sum((e < ncb) ? zs[e] : 0u);
-            base = p.zpre[ncb >> 5] + part;
-            zl = (uint32_t)lane < cnt ? zs[ncb + lane] : 0u;
-        }
-        // the block containing bit `lane` of the word
-        const uint32_t incl = warp_incl_scan(zl);
-        const uint32_t tot = __shfl_sync(0xffffffffu, incl, 31);
-        // each zsize must lie in [1 + ncode, MAXZ]  (ncode = b/4 except the tail block)
-        bool zok = true;
-        if ((uint32_t)lane < cnt) zok = zl >= 2 && zl <= (uint32_t)C::MAXZ;
-        ok = ok && __all_sync(0xffffffffu, zok) && base + tot <= hd.payload_bytes;
-        if ((uint32_t)lane < 32) { s_off[lane] = incl - zl; s_z[lane] = zl; }
-        if (lane == 0) {
-            s_base = base;
-            s_ok = ok;
-            if (!ok) set_corrupt(p.err);
-        }
-    }
-    __syncthreads();
-    if (!s_ok) return;
-    const uint64_t base = s_base;
-    const uint32_t Tb = cnt ? s_off[cnt - 1] + s_z[cnt - 1] : 0;
-    // stage payload bytes [base, base + Tb) with 16-byte loads
-    if (Tb) {
-        const uint8_t* g0 = in + hd.off_pl + base;
-        const uintptr_t A = reinterpret_cast<uintptr_t>(g0) & ~uintptr_t(15);
-        const uintptr_t E = reinterpret_cast<uintptr_t>(g0) + Tb;
+    if (warp == C::NWARP) {
+        // ---------------- producer: per tile, TMA bulk copies of the payload, the 32 mu
+        // values and the tile's zsize window; metadata fetched 32 tiles per round trip
+        const uintptr_t pl = reinterpret_cast<uintptr_t>(in + hd.off_pl);
+        const uintptr_t zsb = reinterpret_cast<uintptr_t>(in + hd.off_zs);
         const uintptr_t lim = reinterpret_cast<uintptr_t>(in) + p.in_bytes;
-        const uint32_t nch = (uint32_t)((E - A + 15) >> 4);
-        for (uint32_t ch = threadIdx.x; ch < nch; ch += C::NT) {
-            const uintptr_t a = A + 16 * (uintptr_t)ch;
-            if (a + 16 <= lim) {
-                *reinterpret_cast<uint4*>(stg + 16 * ch) = ld_stream16(reinterpret_cast<const void*>(a));
-            } else {
-                for (int q = 0; q < 16; q++)
-                    stg[16 * ch + q] = (a + q < lim) ? *reinterpret_cast<const uint8_t*>(a + q) : 0;
+        const uintptr_t lim16 = lim & ~uintptr_t(15);
+        const uint32_t* bm = reinterpret_cast<const uint32_t*>(in + kHeaderBytes);
+        int i = 0;
+        for (uint64_t tb = blockIdx.x; tb < p.nW; tb += 32 * G) {
+            // lane l holds the metadata of tile tb + l*G
+            const uint64_t tl = tb + (uint64_t)lane * G;
+            uint32_t m_word = 0, m_ncb = 0;
+            uint64_t m_base = 0, m_end = 0;
+            if (tl < p.nW) {
+                m_word = bm[tl];
+                m_ncb = p.ncpre[tl];
+                m_base = p.tbase[tl];
+                m_end = p.tbase[tl + 1];
+            }
+            for (int j = 0; j < 32; j++, i++) {
+                const uint64_t t = tb + (uint64_t)j * G;
+                if (t >= p.nW) break;
+                uint32_t word = __shfl_sync(0xffffffffu, m_word, j);
+                const uint32_t ncb = __shfl_sync(0xffffffffu, m_ncb, j);
+                const uint64_t base = __shfl_sync(0xffffffffu, m_base, j);
+                const uint64_t end = __shfl_sync(0xffffffffu, m_end, j);
+                if (t == p.nW - 1 && (p.nB & 31)) word &= (1u << (p.nB & 31)) - 1u;
+                const uint32_t cnt = __popc(word);
+                const int s = i % C::STAGES;
+                mbar_wait(&empty_bar[s], ((i / C::STAGES) & 1) ^ 1);
+                uint8_t* pay = smem + (size_t)s * C::STAGE;
+                uint8_t* mub = pay + C::PAY;
+                const uint64_t Tb = end - base;
+                const bool ok = end >= base && Tb <= (uint64_t)C::TB * C::MAXZ && end <= hd.payload_bytes &&
+                                (uint64_t)ncb + cnt <= hd.nnc;
+                const uintptr_t a0 = pl + base;
+                const uintptr_t A = a0 & ~uintptr_t(15);
+                const uintptr_t E = ok ? ((a0 + Tb + 15) & ~uintptr_t(15)) : A;
+                const uintptr_t Eb = E < lim16 ? E : (lim16 > A ? lim16 : A);  // bulk part inside the buffer
+                const uint32_t bulk = (uint32_t)(Eb - A);
+                const uint64_t k0 = t * C::TB;
+                const bool mu_tma = (k0 + C::TB) <= p.nB;   // full tile of mu values
+                const uintptr_t za = (zsb + 2 * (uint64_t)ncb) & ~uintptr_t(15);
+                const uint32_t zbytes =
+                    (ok && cnt) ? (uint32_t)(((zsb + 2 * ((uint64_t)ncb + cnt) + 15) & ~uintptr_t(15)) - za) : 0u;
+                if (lane == 0) {
+                    mbar_expect_tx(&full_bar[s], bulk + (mu_tma ? (uint32_t)C::MUB : 0u) + zbytes);
+                    if (bulk) tma_load_1d(pay, reinterpret_cast<const void*>(A), bulk, &full_bar[s]);
+                    if (mu_tma) tma_load_1d(mub, in + p.off_mu + k0 * C::W, C::MUB, &full_bar[s]);
+                    if (zbytes) tma_load_1d(&s_zw[s][0], reinterpret_cast<const void*>(za), zbytes, &full_bar[s]);
+                    s_word[s] = word;
+                    s_sb[s] = (uint32_t)(a0 & 15);
+                    s_zo[s] = (uint32_t)((zsb + 2 * (uint64_t)ncb - za) >> 1);
+                    s_ok[s] = ok;
+                    s_T[s] = Tb;
+                }
+                // bytes of the last 16-byte chunk beyond the buffer's 16-byte floor
+                for (uintptr_t a = Eb + lane; a < E; a += 32)
+                    pay[a - A] = a < lim ? *reinterpret_cast<const uint8_t*>(a) : 0;
+                if (!mu_tma) {  // last, partial tile
+                    const U* mus = reinterpret_cast<const U*>(in + p.off_mu);
+                    if (k0 + lane < p.nB) reinterpret_cast<U*>(mub)[lane] = mus[k0 + lane];
+                }
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&full_bar[s]);
             }
         }
+        return;
     }
-    __syncthreads();
-    const int sb = (int)(reinterpret_cast<uintptr_t>(in + hd.off_pl + base) & 15);
-    const U* mus = reinterpret_cast<const U*>(in + p.off_mu);
-#pragma unroll
-    for (int j = 0; j < C::BPW; j++) {
-        const int idx = warp * C::BPW + j;
-        const uint64_t k = tile * kTileBlocks + idx;
-        if (k >= p.nB) break;
-        const int len = (int)umin64(C::B, p.n - k * C::B);
-        const T mu = TR::from(mus[k]);
-        T v[VPL];
-        if (!((word >> idx) & 1u)) {
-#pragma unroll
-            for (int i = 0; i < VPL; i++) v[i] = mu;  // constant block: retrieve with mu
+
+    // ---------------- consumers
+    int i = 0;
+    for (uint64_t t = blockIdx.x; t < p.nW; t += G, i++) {
+        const int s = i % C::STAGES;
+        mbar_wait(&full_bar[s], (i / C::STAGES) & 1);
+        const uint8_t* pay = smem + (size_t)s * C::STAGE;
+        const U* mub = reinterpret_cast<const U*>(pay + C::PAY);
+        const uint32_t word = s_word[s];
+        const uint32_t cnt = __popc(word);
+        const uint32_t zl = (s_ok[s] && (uint32_t)lane < cnt) ? s_zw[s][s_zo[s] + lane] : 0u;
+        const uint32_t zincl = warp_incl_scan(zl);
+        const uint32_t zoff = zincl - zl;  // offset of the lane-th nonconstant block
+        const bool zok = (uint32_t)lane >= cnt || (zl >= 2 && zl <= (uint32_t)C::MAXZ);
+        const bool ok = s_ok[s] && __all_sync(0xffffffffu, zok) && __shfl_sync(0xffffffffu, zincl, 31) == s_T[s];
+        if (!ok) {
+            if (threadIdx.x == 0) set_corrupt(p.err);
         } else {
-            const uint32_t rank = __popc(word & ((1u << idx) - 1u));
-            if (!decode_block<T, VPL>(stg + sb + s_off[rank], s_z[rank], len, mu, v)) {
-                if (lane == 0) set_corrupt(p.err);
-                continue;
+            const int sb = (int)s_sb[s];
+#pragma unroll 1
+            for (int j = 0; j < C::BPW; j++) {
+                const int idx = warp * C::BPW + j;
+                const uint64_t k = t * C::TB + idx;
+                if (k >= p.nB) break;
+                const int len = (int)umin64(C::B, p.n - k * C::B);
+                const T mu = TR::from(mub[idx]);
+                T v[VPL];
+                if (!((word >> idx) & 1u)) {
+#pragma unroll
+                    for (int q = 0; q < VPL; q++) v[q] = mu;  // constant block: retrieve with mu
+                } else {
+                    const uint32_t rank = __popc(word & ((1u << idx) - 1u));
+                    const uint32_t off = __shfl_sync(0xffffffffu, zoff, rank);
+                    const uint32_t z = __shfl_sync(0xffffffffu, zl, rank);
+                    if (!decode_block<T, VPL>(pay + sb + off, z, len, mu, v)) {
+                        if (lane == 0) set_corrupt(p.err);
+                        continue;
+                    }
+                }
+                store_lane<T, VPL>(y, p.n, k, lane, v);
             }
         }
-        store_lane<T, VPL>(y, p.n, k, lane, v);
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&empty_bar[s]);
     }
 }
 

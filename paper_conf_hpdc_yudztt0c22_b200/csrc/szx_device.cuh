@@ -28,6 +28,8 @@ template <> struct Traits<float> {
     static constexpr int W = 4;
     static constexpr int kFloor = 9;   // sign + exponent bits (reading R3)
     static constexpr int kFull = 32;   // "fullbits" (Formula 4) -> raw block
+    static constexpr uint32_t kKeyPInf = 0xFF800000u;  // okey(+Inf); NaN keys lie outside
+    static constexpr uint32_t kKeyNInf = 0x007FFFFFu;  // okey(-Inf)  [kKeyNInf, kKeyPInf]
     __device__ static U bits(float f) { return __float_as_uint(f); }
     __device__ static float from(U u) { return __uint_as_float(u); }
     __device__ static int expo(float f) { return int((__float_as_uint(f) >> 23) & 0xFF) - 127; }
@@ -36,12 +38,18 @@ template <> struct Traits<float> {
     __device__ static float half(float a) { return __fmul_rn(a, 0.5f); }
     __device__ static int clz(U u) { return __clz(u); }
     __device__ static bool isnan_(float f) { return f != f; }
+    // x*0 + acc: stays +-0 while every x is finite, NaN once one is not
+    __device__ static float fma0(float x, float acc) { return __fmaf_rn(x, 0.0f, acc); }
+    __device__ static float fmin_(float a, float b) { return fminf(a, b); }
+    __device__ static float fmax_(float a, float b) { return fmaxf(a, b); }
 };
 template <> struct Traits<double> {
     using U = uint64_t;
     static constexpr int W = 8;
     static constexpr int kFloor = 12;
     static constexpr int kFull = 64;
+    static constexpr uint64_t kKeyPInf = 0xFFF0000000000000ull;
+    static constexpr uint64_t kKeyNInf = 0x000FFFFFFFFFFFFFull;
     __device__ static U bits(double f) { return (U)__double_as_longlong(f); }
     __device__ static double from(U u) { return __longlong_as_double((long long)u); }
     __device__ static int expo(double f) { return int(((U)__double_as_longlong(f) >> 52) & 0x7FF) - 1023; }
@@ -50,21 +58,42 @@ template <> struct Traits<double> {
     __device__ static double half(double a) { return __dmul_rn(a, 0.5); }
     __device__ static int clz(U u) { return __clzll((long long)u); }
     __device__ static bool isnan_(double f) { return f != f; }
+    __device__ static double fma0(double x, double acc) { return __fma_rn(x, 0.0, acc); }
+    __device__ static double fmin_(double a, double b) { return ::fmin(a, b); }
+    __device__ static double fmax_(double a, double b) { return ::fmax(a, b); }
 };
 
 __device__ inline int expo_f64(double e) {
     return int(((uint64_t)__double_as_longlong(e) >> 52) & 0x7FF) - 1023;
 }
 
+// Opaque copy: stops the optimiser from proving that an integer came from a
+// float bitcast and rewriting sign-bit logic as float ops (observed: nvcc
+// turned `u | 0x80000000` into FADD -|x|, which canonicalises NaN payloads).
+__device__ inline uint32_t launder(uint32_t u) {
+    asm("mov.b32 %0, %0;" : "+r"(u));
+    return u;
+}
+__device__ inline uint64_t launder(uint64_t u) {
+    asm("mov.b64 %0, %0;" : "+l"(u));
+    return u;
+}
+
 // Order-preserving unsigned key of a double (total order, -0 < +0).
 __host__ __device__ inline uint64_t dkey(uint64_t bits) {
+#ifdef __CUDA_ARCH__
+    bits = launder(bits);
+#endif
     return (bits & 0x8000000000000000ull) ? ~bits : (bits | 0x8000000000000000ull);
 }
 __host__ __device__ inline uint64_t dkey_inv(uint64_t k) {
     return (k & 0x8000000000000000ull) ? (k & 0x7FFFFFFFFFFFFFFFull) : ~k;
 }
 // Same for the data word (min/max in the data type).
-__device__ inline uint32_t okey(uint32_t u) { return (u & 0x80000000u) ? ~u : (u | 0x80000000u); }
+__device__ inline uint32_t okey(uint32_t u) {
+    u = launder(u);
+    return (u & 0x80000000u) ? ~u : (u | 0x80000000u);
+}
 __device__ inline uint32_t okey_inv(uint32_t k) { return (k & 0x80000000u) ? (k & 0x7FFFFFFFu) : ~k; }
 __device__ inline uint64_t okey(uint64_t u) { return dkey(u); }
 __device__ inline uint64_t okey_inv(uint64_t k) { return dkey_inv(k); }
@@ -76,10 +105,10 @@ __device__ inline double eb_from_range(int mode, double eb_user, const uint64_t*
     if (mode == 0) {
         e = eb_user;
     } else {
-        uint64_t kmin = range_keys[0], kmax = ~range_keys[1];
-        if (range_keys[0] == ~0ull) {
+        if (!range_keys || range_keys[0] == ~0ull) {
             e = 0.0;
         } else {
+            const uint64_t kmin = range_keys[0], kmax = ~range_keys[1];
             double gmin = __longlong_as_double((long long)dkey_inv(kmin));
             double gmax = __longlong_as_double((long long)dkey_inv(kmax));
             e = __dmul_rn(eb_user, __dsub_rn(gmax, gmin));
@@ -119,6 +148,86 @@ __device__ inline uint32_t warp_incl_scan(uint32_t v) {
     return v;
 }
 
+// ---------------------------------------------------------------- byte runs
+// A lane's run of mid-bytes (at most VPL*W bytes) held little-endian in NW
+// 32-bit words, byte 0 first.  Shifts by k <= 8 bytes across the words.
+template <int NW>
+__device__ inline void run_shr(uint32_t (&a)[NW], int k) {
+    // whole words first (k >> 2 is 0, 1 or 2), then the k & 3 remaining bytes;
+    // funnel shifts take their amount mod 32, so 4-byte steps must not reach them
+#pragma unroll
+    for (int r = 0; r < 2; r++) {
+        if (k >= 4) {
+#pragma unroll
+            for (int q = 0; q < NW - 1; q++) a[q] = a[q + 1];
+            a[NW - 1] = 0;
+            k -= 4;
+        }
+    }
+    const int sh = 8 * k;
+#pragma unroll
+    for (int q = 0; q < NW - 1; q++) a[q] = __funnelshift_r(a[q], a[q + 1], sh);
+    a[NW - 1] = sh ? a[NW - 1] >> sh : a[NW - 1];
+}
+template <int NW>
+__device__ inline void run_shl(uint32_t (&a)[NW], int k) {
+#pragma unroll
+    for (int r = 0; r < 2; r++) {
+        if (k >= 4) {
+#pragma unroll
+            for (int q = NW - 1; q > 0; q--) a[q] = a[q - 1];
+            a[0] = 0;
+            k -= 4;
+        }
+    }
+    const int sh = 8 * k;
+#pragma unroll
+    for (int q = NW - 1; q > 0; q--) a[q] = __funnelshift_l(a[q - 1], a[q], sh);
+    a[0] = sh ? a[0] << sh : a[0];
+}
+// Load NW words of bytes starting at an arbitrary shared-memory byte address.
+template <int NW>
+__device__ inline void run_load(const uint8_t* p, uint32_t (&a)[NW]) {
+    const uintptr_t addr = reinterpret_cast<uintptr_t>(p);
+    const uint32_t* w = reinterpret_cast<const uint32_t*>(addr & ~uintptr_t(3));
+    const int sh = 8 * (int)(addr & 3);
+    uint32_t lo = w[0];
+#pragma unroll
+    for (int q = 0; q < NW; q++) {
+        const uint32_t hi = w[q + 1];
+        a[q] = __funnelshift_r(lo, hi, sh);
+        lo = hi;
+    }
+}
+// Store the first len bytes of a run at an arbitrary shared-memory byte
+// address: whole words with 32-bit stores, the partial head / tail words
+// byte by byte (they may be shared with the neighbouring lanes' runs).
+template <int NW>
+__device__ inline void run_store(uint8_t* p, const uint32_t (&a)[NW], int len) {
+    if (len <= 0) return;
+    const uintptr_t addr = reinterpret_cast<uintptr_t>(p);
+    uint32_t* w = reinterpret_cast<uint32_t*>(addr & ~uintptr_t(3));
+    const int h = (int)(addr & 3), e = h + len;
+    const int sh = 8 * h;
+    uint32_t prev = 0;
+#pragma unroll
+    for (int q = 0; q <= NW; q++) {
+        const uint32_t cur = q < NW ? a[q] : 0u;
+        const uint32_t word = sh ? __funnelshift_l(prev, cur, sh) : cur;
+        prev = cur;
+        const int b0 = 4 * q, b1 = 4 * q + 4;   // bytes of this word: [b0, b1)
+        if (b0 >= e) break;
+        if (b0 >= h && b1 <= e) {
+            w[q] = word;
+        } else {
+            uint8_t* bp = reinterpret_cast<uint8_t*>(w + q);
+#pragma unroll
+            for (int j = 0; j < 4; j++)
+                if (b0 + j >= h && b0 + j < e) bp[j] = (uint8_t)(word >> (8 * j));
+        }
+    }
+}
+
 // ---------------------------------------------------------------- memory
 __device__ inline uint64_t ld_relaxed(const uint64_t* p) {
     uint64_t v;
@@ -134,6 +243,46 @@ __device__ inline uint4 ld_stream16(const void* p) {
     asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
                  : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
     return v;
+}
+
+// ---------------------------------------------------------------- TMA / mbarrier
+__device__ inline uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ inline void mbar_init(uint64_t* bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ inline void fence_mbar_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
+__device__ inline void mbar_arrive(uint64_t* bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ inline void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+}
+// raise the expected transaction bytes of the current phase without arriving
+__device__ inline void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.expect_tx.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ inline void mbar_wait(uint64_t* bar, uint32_t parity) {
+    asm volatile(
+        "{\n .reg .pred P1;\n"
+        "WAIT_%=:\n"
+        " mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
+        " @!P1 bra WAIT_%=;\n}\n" ::"r"(smem_u32(bar)),
+        "r"(parity)
+        : "memory");
+}
+// 1-D TMA bulk copy global -> shared, completion counted on an mbarrier
+// (bytes and both addresses multiples of 16).
+__device__ inline void tma_load_1d(void* smem_dst, const void* gsrc, uint32_t bytes, uint64_t* bar) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+            smem_u32(smem_dst)),
+        "l"(gsrc), "r"(bytes), "r"(smem_u32(bar))
+        : "memory");
+}
+// named barrier over the first `nthreads` threads (consumer warps only)
+__device__ inline void bar_sync_named(int id, int nthreads) {
+    asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
 
 // Decoupled look-back (single-pass prefix scan, Merrill & Garland) over
