@@ -86,67 +86,63 @@ __global__ void __launch_bounds__(256) k_block_stats(const T* __restrict__ x, Pl
     U* stats = reinterpret_cast<U*>(p.stats);
     U fmin = ~U(0), fmax = 0;  // finite range (keys), warp-uniform
 
-    for (uint64_t k0 = gw * UNR; k0 < p.nB; k0 += nw * UNR) {
-        T v[UNR][VPL];
-        int cnt[UNR];
+    // one block's keys -> stats and the finite range (all lanes; keys exact,
+    // NaN lies outside [key(-Inf), key(+Inf)] and is detected by k_classify)
+    auto block = [&](const T (&v)[VPL], int cnt, uint64_t k) {
+        U kmn = ~U(0), kmx = 0;
 #pragma unroll
-        for (int u = 0; u < UNR; u++) cnt[u] = (k0 + u < p.nB) ? load_lane<T, VPL>(x, p.n, k0 + u, lane, v[u]) : 0;
-#pragma unroll
-        for (int u = 0; u < UNR; u++) {
-            if (k0 + u >= p.nB) break;
-            // Fast path: float min/max (FMNMX, alu pipe) and a NaN/Inf detector
-            // on the fma pipe (x*0 is NaN iff x is not finite).  Only blocks
-            // whose lanes saw a non-finite value take the exact key path.  The
-            // sign of a zero extreme may differ between the paths; no output
-            // depends on it (DESIGN.md s.3, R1 note).
-            T fmn = v[u][0], fmx = v[u][0], chk = T(0);
-#pragma unroll
-            for (int i = 0; i < VPL; i++) {
-                const T xi = i < cnt[u] ? v[u][i] : v[u][0];
-                fmn = TR::fmin_(fmn, xi);
-                fmx = TR::fmax_(fmx, xi);
-                chk = TR::fma0(xi, chk);
-            }
-            U kmn, kmx;
-            if (__all_sync(0xffffffffu, chk == T(0))) {
-                kmn = cnt[u] ? okey(TR::bits(fmn)) : ~U(0);
-                kmx = cnt[u] ? okey(TR::bits(fmx)) : U(0);
-            } else {
-                kmn = ~U(0);
-                kmx = 0;
+        for (int i = 0; i < VPL; i++) {
+            const U key = okey(TR::bits(v[i]));
+            kmn = i < cnt ? umin_(kmn, key) : kmn;
+            kmx = i < cnt ? umax_(kmx, key) : kmx;
+        }
+        kmn = warp_min(kmn);
+        kmx = warp_max(kmx);
+        if (lane == 0) {
+            stats[2 * k] = kmn;
+            stats[2 * k + 1] = kmx;
+        }
+        if (want_range) {
+            if (kmn > TR::kKeyNInf && kmx < TR::kKeyPInf) {
+                fmin = umin_(fmin, kmn);
+                fmax = umax_(fmax, kmx);
+            } else {  // the block holds +-Inf or NaN: finite extremes value by value (rare)
+                U a = ~U(0), b = 0;
 #pragma unroll
                 for (int i = 0; i < VPL; i++) {
-                    if (i < cnt[u]) {
-                        const U key = okey(TR::bits(v[u][i]));
-                        kmn = umin_(kmn, key);
-                        kmx = umax_(kmx, key);
+                    const U key = okey(TR::bits(v[i]));
+                    if (i < cnt && key > TR::kKeyNInf && key < TR::kKeyPInf) {
+                        a = umin_(a, key);
+                        b = umax_(b, key);
                     }
                 }
+                fmin = umin_(fmin, warp_min(a));
+                fmax = umax_(fmax, warp_max(b));
             }
-            kmn = warp_min(kmn);
-            kmx = warp_max(kmx);
-            if (lane == 0) {
-                stats[2 * (k0 + u)] = kmn;
-                stats[2 * (k0 + u) + 1] = kmx;
-            }
-            if (want_range) {
-                if (kmn > TR::kKeyNInf && kmx < TR::kKeyPInf) {
-                    fmin = umin_(fmin, kmn);
-                    fmax = umax_(fmax, kmx);
-                } else {  // the block holds +-Inf or NaN: finite extremes value by value (rare)
-                    U a = ~U(0), b = 0;
+        }
+    };
+    constexpr int B = 32 * VPL;
+    constexpr int NV = VPL * (int)sizeof(T) / 16;   // 16-byte loads per lane per block
+    const uint64_t nBf = p.n / B;                    // full blocks
+    uint64_t k0 = gw * UNR;
+    // fast path: UNR full blocks per warp, all loads issued first, no bounds checks
+    for (; k0 + UNR <= nBf; k0 += nw * UNR) {
+        const uint4* src = reinterpret_cast<const uint4*>(x + k0 * B) + lane * NV;
+        T v[UNR][VPL];
 #pragma unroll
-                    for (int i = 0; i < VPL; i++) {
-                        const U key = okey(TR::bits(v[u][i]));
-                        if (i < cnt[u] && key > TR::kKeyNInf && key < TR::kKeyPInf) {
-                            a = umin_(a, key);
-                            b = umax_(b, key);
-                        }
-                    }
-                    fmin = umin_(fmin, warp_min(a));
-                    fmax = umax_(fmax, warp_max(b));
-                }
-            }
+        for (int u = 0; u < UNR; u++)
+#pragma unroll
+            for (int q = 0; q < NV; q++) reinterpret_cast<uint4*>(v[u])[q] = ld_stream16(src + u * (B / 4 * sizeof(T) / 4) + q);
+#pragma unroll
+        for (int u = 0; u < UNR; u++) block(v[u], VPL, k0 + u);
+    }
+    // remaining blocks (partial group, tail block): one at a time
+    for (; k0 < p.nB; k0 += nw * UNR) {
+#pragma unroll 1
+        for (int u = 0; u < UNR && k0 + u < p.nB; u++) {
+            T v[VPL];
+            const int cnt = load_lane<T, VPL>(x, p.n, k0 + u, lane, v);
+            block(v, cnt, k0 + u);
         }
     }
     if (want_range) {

@@ -260,6 +260,79 @@ __device__ inline bool decode_block(const uint8_t* src, uint32_t z, int len, T m
     return true;
 }
 
+// Fast path of decode_block for a FULL block (every lane holds VPL values):
+// no per-value tail guards, explicit ld.shared, clamped funnel shifts.
+// src is the shared-memory address of the block payload.
+template <typename T, int VPL>
+__device__ inline bool decode_full(uint32_t src, uint32_t z, T mu, T (&out)[VPL]) {
+    using TR = Traits<T>;
+    using U = typename TR::U;
+    constexpr int W = TR::W;
+    constexpr int NCODE = 8 * VPL;     // (32 * VPL) / 4
+    constexpr int NW = VPL * W / 4;
+    const int lane = threadIdx.x & 31;
+    const int R = (int)lds_u8(src);
+    if (R < TR::kFloor || R > TR::kFull) return false;
+    const bool raw = R >= TR::kFull;
+    const int s = raw ? 0 : ((8 - (R & 7)) & 7);
+    const int req = (R + s) >> 3;
+    // (1) leading numbers: VPL/4 code bytes per lane
+    uint32_t leads = 0;
+#pragma unroll
+    for (int q = 0; q < VPL / 4; q++) leads |= lds_u8(src + 1 + lane * (VPL / 4) + q) << (8 * q);
+    uint32_t m = 0;
+#pragma unroll
+    for (int i = 0; i < VPL; i++) {
+        const int L = (leads >> (2 * i)) & 3;
+        m += req > L ? req - L : 0;
+    }
+    const uint32_t incl = warp_incl_scan(m);
+    if (1u + NCODE + __shfl_sync(0xffffffffu, incl, 31) != z) return false;
+    // (3) this lane's mid-bytes; value i takes the next m_i bytes of the run
+    uint32_t run[NW];
+    run_load_s<NW>(src + 1 + NCODE + incl - m, run);
+    U own[VPL], cmk[VPL];
+    U M = ~U(0), D = 0;  // lane map: c -> (c & M) | D
+#pragma unroll
+    for (int i = 0; i < VPL; i++) {
+        const int L = (leads >> (2 * i)) & 3;
+        const int mi = req > L ? req - L : 0;
+        U bytes;
+        if (W == 4) {
+            bytes = run[0] & (mi >= 4 ? 0xFFFFFFFFu : ((1u << (8 * mi)) - 1u));
+            run_drop4<NW>(run, mi);
+        } else {
+            bytes = ((U)run[0] | ((U)run[1] << 16 << 16)) & (mi >= 8 ? ~U(0) : ((U(1) << (8 * mi)) - U(1)));
+            run_drop4<NW>(run, mi < 4 ? mi : 4);
+            run_drop4<NW>(run, mi > 4 ? mi - 4 : 0);
+        }
+        own[i] = bytes << (8 * (W - req));
+        const int copy = L < req ? L : req;  // (2) bytes copied from the previous value
+        cmk[i] = copy == 0 ? U(0) : (~U(0) << (8 * (W - copy)));
+        M &= cmk[i];
+        D = (D & cmk[i]) | own[i];
+    }
+    // exclusive warp scan of lane maps -> the word carried into this lane (u_{-1} = 0)
+    U cM = M, cD = D;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const U pM = __shfl_up_sync(0xffffffffu, cM, o);
+        const U pD = __shfl_up_sync(0xffffffffu, cD, o);
+        if (lane >= o) { cD = (pD & cM) | cD; cM = pM & cM; }
+    }
+    U prev = __shfl_up_sync(0xffffffffu, cD, 1);
+    if (lane == 0) prev = 0;
+    // (4) combine and overwrite the previous value, (5) left shift, add mu
+#pragma unroll
+    for (int i = 0; i < VPL; i++) {
+        const U w = (prev & cmk[i]) | own[i];
+        prev = w;
+        const U vb = w << s;
+        out[i] = raw ? TR::from(vb) : TR::add(TR::from(vb), mu);
+    }
+    return true;
+}
+
 template <typename T, int VPL>
 __global__ void __launch_bounds__(DecodeCfg<T, VPL>::NT, DecodeCfg<T, VPL>::MINB)
     k_decode(DPlan p, const uint8_t* __restrict__ in, T* __restrict__ y) {
@@ -372,6 +445,35 @@ __global__ void __launch_bounds__(DecodeCfg<T, VPL>::NT, DecodeCfg<T, VPL>::MINB
         const bool ok = s_ok[s] && __all_sync(0xffffffffu, zok) && __shfl_sync(0xffffffffu, zincl, 31) == s_T[s];
         if (!ok) {
             if (threadIdx.x == 0) set_corrupt(p.err);
+        } else if ((t + 1) * C::TB * C::B <= p.n) {
+            // full tile: every block holds B values
+            const uint32_t spay = smem_u32(pay) + s_sb[s];
+            const uint32_t smu = smem_u32(mub) + warp * C::BPW * C::W;
+            uint4* yq = reinterpret_cast<uint4*>(y + (t * C::TB + warp * C::BPW) * C::B + lane * VPL);
+            constexpr int NV = VPL * C::W / 16;       // 16-byte stores per lane per block
+            constexpr int QB = C::B * C::W / 16;      // 16-byte chunks per block
+#pragma unroll 1
+            for (int j = 0; j < C::BPW; j++) {
+                const int idx = warp * C::BPW + j;
+                U mb = lds_u32(smu + j * C::W);
+                if (C::W == 8) mb |= (U)lds_u32(smu + j * C::W + 4) << 16 << 16;
+                const T mu = TR::from(mb);
+                T v[VPL];
+                if (!((word >> idx) & 1u)) {
+#pragma unroll
+                    for (int q = 0; q < VPL; q++) v[q] = mu;  // constant block: retrieve with mu
+                } else {
+                    const uint32_t rank = __popc(word & ((1u << idx) - 1u));
+                    const uint32_t off = __shfl_sync(0xffffffffu, zoff, rank);
+                    const uint32_t z = __shfl_sync(0xffffffffu, zl, rank);
+                    if (!decode_full<T, VPL>(spay + off, z, mu, v)) {
+                        if (lane == 0) set_corrupt(p.err);
+                        continue;
+                    }
+                }
+#pragma unroll
+                for (int q = 0; q < NV; q++) yq[j * QB + q] = reinterpret_cast<const uint4*>(v)[q];
+            }
         } else {
             const int sb = (int)s_sb[s];
 #pragma unroll 1

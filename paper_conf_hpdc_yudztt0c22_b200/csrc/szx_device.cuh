@@ -148,6 +148,49 @@ __device__ inline uint32_t warp_incl_scan(uint32_t v) {
     return v;
 }
 
+// ---------------------------------------------------------------- shared memory
+// Explicit ld.shared (generic pointers into the staging buffers otherwise
+// compile to generic LD.E).  volatile: keeps them after the mbarrier waits.
+__device__ inline uint32_t lds_u8(uint32_t a) {
+    uint32_t v;
+    asm volatile("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(a));
+    return v;
+}
+__device__ inline uint32_t lds_u32(uint32_t a) {
+    uint32_t v;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
+    return v;
+}
+// Run of bytes starting at an arbitrary shared address, realigned into NW words.
+template <int NW>
+__device__ inline void run_load_s(uint32_t a, uint32_t (&r)[NW]) {
+    const uint32_t base = a & ~3u, sh = 8 * (a & 3u);
+    uint32_t lo = lds_u32(base);
+#pragma unroll
+    for (int q = 0; q < NW; q++) {
+        const uint32_t hi = lds_u32(base + 4 * (q + 1));
+        r[q] = __funnelshift_r(lo, hi, sh);
+        lo = hi;
+    }
+}
+// Drop the first k (0..4) bytes of a run: clamped funnel shifts (a shift of
+// 32 yields the next word), no data-dependent word moves.
+template <int NW>
+__device__ inline void run_drop4(uint32_t (&a)[NW], uint32_t k) {
+    const uint32_t sh = 8 * k;
+#pragma unroll
+    for (int q = 0; q < NW - 1; q++) a[q] = __funnelshift_rc(a[q], a[q + 1], sh);
+    a[NW - 1] = __funnelshift_rc(a[NW - 1], 0u, sh);
+}
+// Insert k (0..4) zero bytes at the front of a run.
+template <int NW>
+__device__ inline void run_push4(uint32_t (&a)[NW], uint32_t k) {
+    const uint32_t sh = 8 * k;
+#pragma unroll
+    for (int q = NW - 1; q > 0; q--) a[q] = __funnelshift_lc(a[q - 1], a[q], sh);
+    a[0] = __funnelshift_lc(0u, a[0], sh);
+}
+
 // ---------------------------------------------------------------- byte runs
 // A lane's run of mid-bytes (at most VPL*W bytes) held little-endian in NW
 // 32-bit words, byte 0 first.  Shifts by k <= 8 bytes across the words.
