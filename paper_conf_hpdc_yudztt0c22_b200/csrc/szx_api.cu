@@ -103,14 +103,14 @@ uint64_t cdiv(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
 // ------------------------------------------------------------ compress layout
 struct CLayout {
     uint64_t nB, nW, nTB, nTC;
-    uint64_t off_keys, off_zero, zero_bytes, off_scal, off_stats, off_nclist, off_nckeys, total;
+    uint64_t off_keys, off_zero, zero_bytes, off_scal, off_stats, off_nclist, off_nckeys, off_ncR, off_gbase, total;
 };
 CLayout clayout(uint64_t n, int W, uint32_t b) {
     CLayout L{};
     L.nB = cdiv(n, b);
     L.nW = cdiv(L.nB, 32);
     L.nTB = cdiv(L.nB, kClassifyBlocks);
-    L.nTC = cdiv(L.nB, 16);  // encode tiles hold >= 16 nonconstant blocks
+    L.nTC = cdiv(cdiv(L.nB, kWriteTile), 256);  // k_zscan CTAs
     L.off_keys = 0;
     L.off_zero = 16;
     L.zero_bytes = al16(16 + 8 * L.nTB + 8 * L.nTC);
@@ -118,7 +118,9 @@ CLayout clayout(uint64_t n, int W, uint32_t b) {
     L.off_stats = L.off_scal + 32;
     L.off_nclist = al16(L.off_stats + 2ull * W * L.nB);
     L.off_nckeys = al16(L.off_nclist + 4 * L.nB + 4);
-    L.total = al16(L.off_nckeys + 2ull * W * L.nB + 16) + 256;  // +16: TMA reads whole 16 B chunks
+    L.off_ncR = al16(L.off_nckeys + 2ull * W * L.nB + 16);
+    L.off_gbase = al16(L.off_ncR + L.nB);
+    L.total = al16(L.off_gbase + 8 * (cdiv(L.nB, kWriteTile) + 2)) + 256;
     return L;
 }
 
@@ -139,7 +141,9 @@ Plan make_plan(const CLayout& L, uint8_t* ws, uint64_t n, szx_dtype_t dt, szx_eb
     p.total = reinterpret_cast<uint64_t*>(ws + L.off_scal + 16);
     p.stats = ws + L.off_stats;
     p.nclist = reinterpret_cast<uint32_t*>(ws + L.off_nclist);
-    p.nckeys = ws + L.off_nckeys;
+    p.ncmu = ws + L.off_nckeys;
+    p.ncR = ws + L.off_ncR;
+    p.gbase = reinterpret_cast<uint64_t*>(ws + L.off_gbase);
     return p;
 }
 
@@ -158,7 +162,8 @@ template <typename T, int VPL>
 void set_smem_attrs() {
     static bool done = false;
     if (done) return;
-    cudaFuncSetAttribute(k_encode<T, VPL>, cudaFuncAttributeMaxDynamicSharedMemorySize, EncodeCfg<T, VPL>::SMEM);
+    cudaFuncSetAttribute(k_enc_write<T, VPL>, cudaFuncAttributeMaxDynamicSharedMemorySize, WriteCfg<T, VPL>::SMEM);
+    cudaFuncSetAttribute(k_enc_size<T, VPL>, cudaFuncAttributeMaxDynamicSharedMemorySize, SizeCfg<T, VPL>::SMEM);
     cudaFuncSetAttribute(k_decode<T, VPL>, cudaFuncAttributeMaxDynamicSharedMemorySize, DecodeCfg<T, VPL>::SMEM);
     done = true;
 }
@@ -182,24 +187,30 @@ void enqueue_stats(const void* d_in, const Plan& p, int want_range, cudaStream_t
     });
 }
 
-// classify (ticketed look-back tiles) then the persistent encoder: one wave of
-// CTAs, all co-resident (required by the look-back across round-robin tiles)
+// classify, then the encoder: size pass (z_k and R per nonconstant block),
+// offset scan, write pass.  Grids are sized for the worst case (every block
+// nonconstant); CTAs beyond the device-side count exit at once.
 template <typename T, int VPL>
 void enqueue_encode(const void* d_in, const Plan& p, const CLayout& L, uint8_t* out, cudaStream_t s) {
     set_smem_attrs<T, VPL>();
     launch("k_classify", s, [&] { k_classify<T><<<(unsigned)L.nTB, 256, 0, s>>>(p, out); });
-    using C = EncodeCfg<T, VPL>;
     static int occ = 0;
     if (!occ) {
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_encode<T, VPL>, C::NT, C::SMEM);
-        if (occ <= 0) occ = 1;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_enc_size<T, VPL>, 256, SizeCfg<T, VPL>::SMEM);
+        if (occ <= 0) occ = 2;
     }
-    uint64_t grid = cdiv(L.nB, C::TB);
+    uint64_t grid = cdiv(L.nB, 8);
     const uint64_t cap = (uint64_t)sm_count() * occ;
     if (grid > cap) grid = cap;
     if (grid == 0) grid = 1;
-    launch("k_encode", s, [&] {
-        k_encode<T, VPL><<<(unsigned)grid, C::NT, C::SMEM, s>>>(static_cast<const T*>(d_in), p, out);
+    launch("k_enc_size", s, [&] {
+        k_enc_size<T, VPL><<<(unsigned)grid, 256, SizeCfg<T, VPL>::SMEM, s>>>(static_cast<const T*>(d_in), p, out);
+    });
+    launch("k_zscan", s, [&] { k_zscan<Traits<T>::W><<<(unsigned)L.nTC, 256, 0, s>>>(p, out); });
+    using C = WriteCfg<T, VPL>;
+    launch("k_enc_write", s, [&] {
+        k_enc_write<T, VPL><<<(unsigned)cdiv(L.nB, kWriteTile), 256, C::SMEM, s>>>(static_cast<const T*>(d_in), p,
+                                                                                   out);
     });
 }
 

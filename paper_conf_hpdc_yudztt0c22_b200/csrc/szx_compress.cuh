@@ -46,7 +46,9 @@ struct Plan {
     uint64_t* status_c;        // encode look-back, init 0
     void* stats;               // 2 keys per block (min, max)
     uint32_t* nclist;          // ids of the nonconstant blocks, in block order
-    void* nckeys;              // their (min, max) keys, same order
+    void* ncmu;                // their mu (bits), same order
+    uint8_t* ncR;              // classify: R_init | proven << 7; size pass: final R
+    uint64_t* gbase;           // payload offset of each write tile (+ total)
     double* eb_abs;            // [1]
     uint64_t* nnc;             // [1]
     uint64_t* total;           // [1] stream bytes (output of the call)
@@ -182,24 +184,57 @@ __device__ inline int initial_R(T r, int pe, int r_bias) {
 template <typename T>
 struct BlockClass {
     bool nan, constant;
-    T mu, r;
+    T mu, r, mn, mx;
 };
 template <typename T>
-__device__ inline BlockClass<T> classify(typename Traits<T>::U kmn, typename Traits<T>::U kmx, double eb) {
+__device__ inline BlockClass<T> classify(typename Traits<T>::U kmn, typename Traits<T>::U kmx, double eb,
+                                         bool test_constant = true) {
     using TR = Traits<T>;
     BlockClass<T> c;
     c.nan = kmn < TR::kKeyNInf || kmx > TR::kKeyPInf;  // R14
     c.constant = false;
-    c.mu = T(0);
-    c.r = T(0);
+    c.mu = c.r = c.mn = c.mx = T(0);
     if (!c.nan) {
-        const T mn = TR::from(okey_inv(kmn)), mx = TR::from(okey_inv(kmx));
-        c.r = TR::half(TR::sub(mx, mn));   // radius r_k (R1)
-        c.mu = TR::add(mn, c.r);           // mu_k = mn + r (R1)
-        c.constant = ((double)c.r <= eb) && (__dsub_rn((double)mx, (double)c.mu) <= eb) &&
-                     (__dsub_rn((double)c.mu, (double)mn) <= eb);  // R2 guard
+        c.mn = TR::from(okey_inv(kmn));
+        c.mx = TR::from(okey_inv(kmx));
+        c.r = TR::half(TR::sub(c.mx, c.mn));   // radius r_k (R1)
+        c.mu = TR::add(c.mn, c.r);             // mu_k = mn + r (R1)
+        if (test_constant)
+            c.constant = ((double)c.r <= eb) && (__dsub_rn((double)c.mx, (double)c.mu) <= eb) &&
+                         (__dsub_rn((double)c.mu, (double)c.mn) <= eb);  // R2 guard
     }
     return c;
+}
+
+// 2^n as a double for n in [-1074, 1023] (exact; subnormal below -1022)
+__device__ inline double pow2d(int n) {
+    if (n >= -1022) return __longlong_as_double((long long)(n + 1023) << 52);
+    return n >= -1074 ? __longlong_as_double(1ll << (n + 1074)) : 0.0;
+}
+
+// Per-block proof that the R2 per-element check cannot fail for R kept bits
+// (DESIGN.md s.3, R2): with E_v <= p(r) and k = R - floor kept mantissa bits,
+//   |x - x'| < 2^(p(r)-k) [truncation] + 2^(E_v-P) [v = fl(x-mu)]
+//            + 2^(E_x'-P) [x' = fl(v'+mu)]  <=  2^p(e) + slack = e
+// when p(r)-k <= p(e) and 2*max(2nd, 3rd term) <= slack = e - 2^p(e) (exact).
+// If it does not hold the kernel evaluates the check value by value, exactly
+// like the oracle, so the stream never depends on this shortcut.
+template <typename T>
+__device__ inline bool guard_proven(const BlockClass<T>& c, double eb, int pe, int R) {
+    using TR = Traits<T>;
+    constexpr int P = sizeof(T) == 4 ? 24 : 53;          // significand bits
+    constexpr int EMIN = sizeof(T) == 4 ? -126 : -1022;  // smallest normal exponent
+    const int pr = TR::expo(c.r);
+    if (c.nan || pr < EMIN || pr >= (sizeof(T) == 4 ? 128 : 1024)) return false;
+    const T v1 = fabs(TR::sub(c.mx, c.mu)), v2 = fabs(TR::sub(c.mn, c.mu));
+    if (TR::expo(v1 > v2 ? v1 : v2) > pr) return false;
+    if (pr - (R - TR::kFloor) > pe) return false;
+    const T a1 = fabs(c.mn), a2 = fabs(c.mx);
+    int ex = TR::expo(a1 > a2 ? a1 : a2) + 1;
+    ex = ex < EMIN ? EMIN : ex;
+    const int t2 = (pr > EMIN ? pr : EMIN) - P, t3 = ex - P;
+    const double slack = __dsub_rn(eb, pow2d(pe));
+    return pow2d((t2 > t3 ? t2 : t3) + 1) <= slack;
 }
 
 __device__ inline void write_header(uint8_t* out, const Plan& p, double eb, uint64_t nnc, uint64_t pbytes) {
@@ -236,17 +271,26 @@ __global__ void __launch_bounds__(256) k_classify(Plan p, uint8_t* __restrict__ 
     U* mus = reinterpret_cast<U*>(out + p.off_mu);
 
     uint32_t ncmask = 0;
+    U rmu[8];
+    uint32_t rrec[2] = {0u, 0u};  // per j: R_init | guard_proven << 7 (one byte each)
 #pragma unroll
     for (int j = 0; j < 8; j++) {
         const uint64_t k = base + j * 256 + threadIdx.x;
         bool nc = false;
+        rmu[j] = 0;
         if (k < p.nB) {
             BlockClass<T> c = classify<T>(stats[2 * k], stats[2 * k + 1], eb);
             T mu = c.mu;
             if (!c.constant) {
                 nc = true;
-                if (c.nan || initial_R<T>(c.r, pe, p.r_bias) >= TR::kFull) mu = T(0);  // raw: mu = +0 (R15)
+                // the per-block scalar work of the encoder is done here once per
+                // block (one thread) instead of once per lane of the encoding warp
+                const int R = c.nan ? TR::kFull : initial_R<T>(c.r, pe, p.r_bias);
+                if (R >= TR::kFull) mu = T(0);  // raw: mu = +0 (R15)
+                const bool proven = R < TR::kFull && guard_proven<T>(c, eb, pe, R);
+                rrec[j >> 2] |= (uint32_t)(R | (proven ? 0x80 : 0)) << (8 * (j & 3));
             }
+            rmu[j] = TR::bits(mu);
             mus[k] = TR::bits(mu);
         }
         const uint32_t word = __ballot_sync(0xffffffffu, nc);
@@ -289,7 +333,7 @@ __global__ void __launch_bounds__(256) k_classify(Plan p, uint8_t* __restrict__ 
     }
     __syncthreads();
     const uint64_t G = s_base;
-    U* nckeys = reinterpret_cast<U*>(p.nckeys);
+    U* ncmu = reinterpret_cast<U*>(p.ncmu);
 #pragma unroll
     for (int j = 0; j < 8; j++) {
         const bool nc = (ncmask >> j) & 1u;
@@ -298,8 +342,8 @@ __global__ void __launch_bounds__(256) k_classify(Plan p, uint8_t* __restrict__ 
             const uint64_t k = base + j * 256 + threadIdx.x;
             const uint64_t idx = G + s_pre[j * 8 + warp] + __popc(word & ((1u << lane) - 1u));
             p.nclist[idx] = (uint32_t)k;
-            nckeys[2 * idx] = stats[2 * k];  // keys in nonconstant order (read by TMA in k_encode)
-            nckeys[2 * idx + 1] = stats[2 * k + 1];
+            ncmu[idx] = rmu[j];
+            p.ncR[idx] = (uint8_t)(rrec[j >> 2] >> (8 * (j & 3)));
         }
     }
 }
@@ -315,35 +359,36 @@ struct LaneCode {
 };
 
 template <typename T, int VPL>
-__device__ inline void encode_block(const T (&xv)[VPL], int cnt, int len, const BlockClass<T>& c,
-                                    double eb, int pe, int r_bias, typename Traits<T>::U (&u)[VPL],
-                                    LaneCode& lc) {
+__device__ inline void encode_block(const T (&xv)[VPL], int cnt, int len, T mu, int R, bool proven,
+                                    double eb, typename Traits<T>::U (&u)[VPL], LaneCode& lc) {
     using TR = Traits<T>;
     using U = typename TR::U;
     constexpr int W = TR::W;
     const int lane = threadIdx.x & 31;
-    int R = c.nan ? TR::kFull : initial_R<T>(c.r, pe, r_bias);
-    T mu = c.mu;
     int s, req;
     bool raw;
+    bool check = !proven;
     for (;;) {
         raw = R >= TR::kFull;
         if (raw) { R = TR::kFull; mu = T(0); }
         s = raw ? 0 : ((8 - (R & 7)) & 7);
         req = (R + s) >> 3;
-        const U keep = raw ? ~U(0) : ~((U(1) << (8 * W - R)) - U(1));
+#pragma unroll
+        for (int i = 0; i < VPL; i++)  // v_i = d_i - mu, then the Solution C shift
+            u[i] = (raw ? TR::bits(xv[i]) : TR::bits(TR::sub(xv[i], mu))) >> s;
+        if (raw || !check) break;
+        // R2 guard (warp-uniform branch): reconstruct exactly as the decoder does
+        // and check Formula 1 value by value
+        const U keep = ~((U(1) << (8 * W - R)) - U(1));
         bool ok = true;
 #pragma unroll
         for (int i = 0; i < VPL; i++) {
-            const U vb = raw ? TR::bits(xv[i]) : TR::bits(TR::sub(xv[i], mu));  // v_i = d_i - mu
-            u[i] = vb >> s;                                                     // Solution C shift
-            if (!raw && i < cnt) {
-                // R2 guard: reconstruct exactly as the decoder does, check Formula 1
-                const T xp = TR::add(TR::from(vb & keep), mu);
+            if (i < cnt) {
+                const T xp = TR::add(TR::from((u[i] << s) & keep), mu);
                 ok &= fabs(__dsub_rn((double)xv[i], (double)xp)) <= eb;
             }
         }
-        if (raw || __all_sync(0xffffffffu, ok)) break;
+        if (__all_sync(0xffffffffu, ok)) break;
         R += 1;
     }
     // identical leading bytes vs the previous value (u_{-1} = 0, R6)
@@ -410,220 +455,349 @@ __device__ inline void pack_block(const typename Traits<T>::U (&u)[VPL], const L
     run_store<NW>(dst + 1 + ncode + lc.mexcl, run, rlen);
 }
 
-// ------------------------------------------------------------------ K2+K3+K4
+// Fast path of pack_block for a FULL block: run assembled with clamped
+// funnel shifts, written with predicated 32-bit / byte shared stores.
+// dst is the shared-memory address of the block payload.
 template <typename T, int VPL>
-struct EncodeCfg {
-    static constexpr int W = Traits<T>::W;
-    static constexpr int B = 32 * VPL;
-    static constexpr int BW = B * W;                     // bytes per full block
-    static constexpr int TB = VPL == 4 ? 32 : 16;        // nonconstant blocks per tile
-    static constexpr int NWARP = 8;                      // consumer warps
-    static constexpr int NC = NWARP * 32;                // consumer threads
-    static constexpr int BPW = TB / NWARP;               // blocks per consumer warp
-    static constexpr int NT = NC + 32;                   // + 1 producer warp
-    static constexpr int STAGES = W == 4 ? 3 : 2;
-    static constexpr int MAXZ = 1 + B / 4 + W * B;       // max z_k
-    static constexpr int KEYB = TB * 2 * W;              // (min, max) keys of a tile
-    static constexpr int RING = STAGES * (TB * BW + KEYB);
-    static constexpr int STG = (16 + TB * MAXZ + 16 + 15) / 16 * 16;
-    static constexpr int SMEM = RING + STG;
-    static constexpr int MINB = W == 4 ? 3 : 2;          // CTAs per SM (register budget)
-};
-
-// Persistent encoder.  Tiles of TB nonconstant blocks are dealt round-robin
-// (tile t -> CTA t mod G).  Payload offsets: every tile publishes its
-// aggregate z-sum; tile t's exclusive prefix is this CTA's own previous
-// inclusive prefix (tile t-G) plus the G-1 aggregates in between, read in
-// parallel by all consumer threads -- one L2 round trip instead of a look-back
-// walk across a whole round of concurrently running tiles.
-template <typename T, int VPL>
-__global__ void __launch_bounds__(EncodeCfg<T, VPL>::NT, EncodeCfg<T, VPL>::MINB)
-    k_encode(const T* __restrict__ x, Plan p, uint8_t* __restrict__ out) {
+__device__ inline void pack_full(const typename Traits<T>::U (&u)[VPL], const LaneCode& lc, uint32_t dst) {
     using TR = Traits<T>;
     using U = typename TR::U;
-    using C = EncodeCfg<T, VPL>;
     constexpr int W = TR::W;
-    extern __shared__ __align__(128) uint8_t smem[];
-    uint8_t* stg = smem + C::RING;
-    __shared__ __align__(8) uint64_t full_bar[C::STAGES], empty_bar[C::STAGES];
-    __shared__ uint32_t s_blk[C::STAGES][C::TB];
-    __shared__ uint32_t s_z[2][C::TB];
-    __shared__ uint64_t s_part[2][C::NWARP];
-    __shared__ uint32_t s_lc[C::TB][32];  // per block and lane: leads | mid-byte offset << 16
-    __shared__ uint8_t s_R[C::TB];
+    constexpr int NCODE = 8 * VPL;
+    constexpr int NW = VPL * W / 4;
+    const int lane = threadIdx.x & 31;
+    const bool raw = lc.R >= TR::kFull;
+    const int s = raw ? 0 : ((8 - (lc.R & 7)) & 7);
+    const int req = (lc.R + s) >> 3;
+    sts_u8_if(lane == 0, dst, (uint32_t)lc.R);
+#pragma unroll
+    for (int q = 0; q < VPL / 4; q++) sts_u8_if(true, dst + 1 + lane * (VPL / 4) + q, lc.leads >> (8 * q));
+    uint32_t run[NW];
+#pragma unroll
+    for (int q = 0; q < NW; q++) run[q] = 0;
+    int rlen = 0;
+#pragma unroll
+    for (int i = VPL - 1; i >= 0; i--) {
+        const int L = (lc.leads >> (2 * i)) & 3;
+        const int mi = req > L ? req - L : 0;
+        // drop the L lead bytes at the top, then bring the mid-bytes down
+        const U hi = u[i] << (8 * L);
+        const int rs = 8 * (W - req + L);
+        if (W == 4) {
+            run_push4<NW>(run, mi);
+            run[0] |= __funnelshift_rc((uint32_t)hi, 0u, rs);   // clamped: rs >= 32 gives 0
+        } else {
+            run_push4<NW>(run, mi > 4 ? mi - 4 : 0);
+            run_push4<NW>(run, mi < 4 ? mi : 4);
+            const uint64_t bm = rs >= 64 ? 0ull : ((uint64_t)hi >> rs);
+            run[0] |= (uint32_t)bm;
+            run[1] |= (uint32_t)(bm >> 32);
+        }
+        rlen += mi;
+    }
+    run_store_s<NW>(dst + 1 + NCODE + lc.mexcl, run, rlen);
+}
 
+// ------------------------------------------------------------------ K2 size pass
+// For every nonconstant block (compacted list): encode (Formula 4 R, R2
+// guard / escalation), write z_k into the stream's zsize section and the
+// final R into the workspace.  A warp owns a contiguous run of the list; it
+// fetches the block metadata 32 blocks per round trip and stages the values
+// of NB blocks at a time in shared memory with cp.async, double-buffered, so
+// the loads of batch b+1 overlap the encoding of batch b.
+template <typename T, int VPL>
+struct SizeCfg {
+    static constexpr int W = Traits<T>::W;
+    static constexpr int B = 32 * VPL;
+    static constexpr int BW = B * W;
+    static constexpr int QV = VPL * W / 16;      // 16-byte chunks per lane per block
+    static constexpr int NB = 4;                 // blocks per batch
+    static constexpr int WARP_BYTES = 2 * NB * BW;
+    static constexpr int SMEM = 8 * WARP_BYTES;
+};
+
+template <typename T, int VPL>
+__global__ void __launch_bounds__(256) k_enc_size(const T* __restrict__ x, Plan p, uint8_t* __restrict__ out) {
+    using TR = Traits<T>;
+    using U = typename TR::U;
+    using C = SizeCfg<T, VPL>;
+    constexpr int W = TR::W;
+    constexpr int B = C::B;
+    extern __shared__ __align__(16) uint8_t smem[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const uint64_t nnc = *p.nnc;
-    const uint64_t ntiles = (nnc + C::TB - 1) / C::TB;
-    const uint64_t G = gridDim.x;
-    if (threadIdx.x == 0) {
-        for (int s = 0; s < C::STAGES; s++) {
-            mbar_init(&full_bar[s], 1);
-            mbar_init(&empty_bar[s], C::NWARP);
-        }
-        fence_mbar_init();
-    }
-    __syncthreads();
-    const bool tail_partial = (p.n % C::B) != 0;
-    auto slot_of = [&](int s, int bi) { return smem + (size_t)s * (C::TB * C::BW + C::KEYB) + (size_t)bi * C::BW; };
-    auto keys_of = [&](int s) {
-        return reinterpret_cast<const U*>(smem + (size_t)s * (C::TB * C::BW + C::KEYB) + C::TB * C::BW);
-    };
-
-    if (warp == C::NWARP) {
-        // ---------------- producer: TMA the nonconstant blocks (and their keys) of each tile
-        const uint8_t* nckeys = reinterpret_cast<const uint8_t*>(p.nckeys);
-        uint64_t t = blockIdx.x;
-        uint32_t kcur = 0;
-        if (t < ntiles && lane < C::TB && t * C::TB + lane < nnc) kcur = p.nclist[t * C::TB + lane];
-        for (int i = 0; t < ntiles; t += G, i++) {
-            const int s = i % C::STAGES;
-            // prefetch the next tile's block ids while this one is issued
-            uint32_t knext = 0;
-            const uint64_t tn = t + G;
-            if (tn < ntiles && lane < C::TB && tn * C::TB + lane < nnc) knext = p.nclist[tn * C::TB + lane];
-            mbar_wait(&empty_bar[s], ((i / C::STAGES) & 1) ^ 1);
-            const uint64_t nc = t * C::TB + lane;
-            const bool act = lane < C::TB && nc < nnc;
-            const bool tail = act && tail_partial && (uint64_t)kcur == p.nB - 1;
-            const uint32_t bytes = (act && !tail) ? (uint32_t)C::BW : 0u;  // the partial tail block is read directly
-            if (lane < C::TB) s_blk[s][lane] = kcur;
-            const uint32_t ntile = (uint32_t)umin64(C::TB, nnc - t * C::TB);
-            const uint32_t kbytes = (ntile * 2 * W + 15) & ~15u;  // nckeys has >= 16 B of slack
-            const uint32_t total = warp_sum(bytes) + kbytes;
-            __syncwarp();
-            if (lane == 0) {
-                mbar_expect_tx(&full_bar[s], total);
-                tma_load_1d(smem + (size_t)s * (C::TB * C::BW + C::KEYB) + C::TB * C::BW,
-                            nckeys + t * (uint64_t)C::KEYB, kbytes, &full_bar[s]);
-            }
-            if (bytes) tma_load_1d(slot_of(s, lane), x + (uint64_t)kcur * C::B, bytes, &full_bar[s]);
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&full_bar[s]);
-            kcur = knext;
-        }
-        return;
-    }
-
-    // ---------------- consumers
     const double eb = *p.eb_abs;
-    const int pe = expo_f64(eb);
     const uint64_t off_zs = p.off_mu + al16((uint64_t)W * p.nB);
-    const uint64_t off_pl = off_zs + al16(2 * nnc);
     uint16_t* zsize = reinterpret_cast<uint16_t*>(out + off_zs);
     U* mus = reinterpret_cast<U*>(out + p.off_mu);
-    uint64_t incl_own = 0;  // inclusive payload prefix of this CTA's previous tile (t - G)
-    int i = 0;
-    for (uint64_t t = blockIdx.x; t < ntiles; t += G, i++) {
-        const int s = i % C::STAGES, par = i & 1;
-        mbar_wait(&full_bar[s], (i / C::STAGES) & 1);
-        const U* keys = keys_of(s);
-        // encode one block at a time; the shifted words go back into the
-        // block's ring slot (same size as the input) and the lane state into
-        // shared memory until packing
-#pragma unroll 1
-        for (int j = 0; j < C::BPW; j++) {
-            const int bi = warp * C::BPW + j;
-            const uint64_t nc = t * C::TB + bi;
-            uint4* slot = reinterpret_cast<uint4*>(slot_of(s, bi)) + lane * (VPL * W / 16);
-            uint32_t z = 0;
-            if (nc < nnc) {
-                const uint32_t k = s_blk[s][bi];
-                const BlockClass<T> cls = classify<T>(keys[2 * bi], keys[2 * bi + 1], eb);
-                T xv[VPL];
-                int cnt = VPL;
-                if (tail_partial && (uint64_t)k == p.nB - 1) {
-                    cnt = load_lane<T, VPL>(x, p.n, k, lane, xv);
-                } else {
+    const U* ncmu = reinterpret_cast<const U*>(p.ncmu);
+    const uint64_t gw = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    const uint64_t chunk = ((nnc + nw - 1) / nw + C::NB - 1) / C::NB * C::NB;
+    const uint64_t c0 = gw * chunk, c1 = umin64(nnc, c0 + chunk);
+    const uint32_t sbuf = smem_u32(smem) + warp * C::WARP_BYTES;
+    const uint64_t nBfull = p.n / B;
+    for (uint64_t g0 = c0; g0 < c1; g0 += 32) {
+        // metadata of 32 blocks: lane l holds block g0 + l
+        const uint64_t gi = g0 + lane;
+        const bool gv = gi < c1;
+        const uint32_t mk = gv ? p.nclist[gi] : 0u;
+        const U mmu = gv ? ncmu[gi] : U(0);
+        const uint32_t mrec = gv ? p.ncR[gi] : 0u;
+        const int nbat = (int)((umin64(32, c1 - g0) + C::NB - 1) / C::NB);
+        auto issue = [&](int b) {
+            const uint32_t st = sbuf + (b & 1) * C::NB * C::BW;
 #pragma unroll
-                    for (int q = 0; q < VPL * W / 16; q++) reinterpret_cast<uint4*>(xv)[q] = slot[q];
-                }
-                const int len = (int)umin64(C::B, p.n - (uint64_t)k * C::B);
-                U u[VPL];
-                LaneCode lc;
-                encode_block<T, VPL>(xv, cnt, len, cls, eb, pe, p.r_bias, u, lc);
+            for (int j = 0; j < C::NB; j++) {
+                const int l = b * C::NB + j;
+                const uint32_t k = __shfl_sync(0xffffffffu, mk, l);
+                if (g0 + l < c1 && k < nBfull) {
+                    const T* src = x + (uint64_t)k * B + lane * VPL;
 #pragma unroll
-                for (int q = 0; q < VPL * W / 16; q++) slot[q] = reinterpret_cast<const uint4*>(u)[q];
-                s_lc[bi][lane] = lc.leads | (lc.mexcl << 16);
-                z = lc.z;
-                if (lane == 0) {
-                    s_R[bi] = (uint8_t)lc.R;
-                    if (lc.R >= TR::kFull) mus[k] = 0;  // raw by escalation: mu = +0 (R15)
+                    for (int q = 0; q < C::QV; q++)
+                        cp_async16(st + j * C::BW + (lane * C::QV + q) * 16, src + q * (16 / W));
                 }
             }
-            if (lane == 0) s_z[par][bi] = z;
-        }
-        bar_sync_named(1, C::NC);
-
-        // tile scan (every warp, redundantly) and publication of the aggregate
-        const uint32_t zl = lane < C::TB ? s_z[par][lane] : 0u;
-        const uint32_t zincl = warp_incl_scan(zl);
-        const uint32_t agg = __shfl_sync(0xffffffffu, zincl, 31);
-        if (threadIdx.x == 0) st_relaxed(&p.status_c[t], kFlagAgg | agg);
-        // sum of the aggregates of tiles (t - G, t): spin until each is published
-        uint64_t part = 0;
-        const uint64_t span = t < G ? t : G - 1;
-        for (uint64_t d = threadIdx.x + 1; d <= span; d += C::NC) {
-            uint64_t v;
-            while (((v = ld_relaxed(&p.status_c[t - d])) & kFlagAgg) == 0) {
-            }
-            part += v & kValueMask;
-        }
-        part = warp_sum64(part);
-        if (lane == 0) s_part[par][warp] = part;
-        bar_sync_named(1, C::NC);
-        uint64_t excl = t < G ? 0 : incl_own;
-#pragma unroll
-        for (int w = 0; w < C::NWARP; w++) excl += s_part[par][w];
-        incl_own = excl + agg;
-        if (t == ntiles - 1 && threadIdx.x == 0) {
-            reinterpret_cast<uint64_t*>(out)[6] = incl_own;  // header: payload bytes
-            *p.total = off_pl + incl_own;
-        }
-        const int sb = (int)(excl & 15);
-
-        // pack payloads into shared memory, write zsize
-#pragma unroll 1
-        for (int j = 0; j < C::BPW; j++) {
-            const int bi = warp * C::BPW + j;
-            const uint64_t nc = t * C::TB + bi;
-            const uint32_t zo = __shfl_sync(0xffffffffu, zincl - zl, bi);
-            const uint32_t zb = __shfl_sync(0xffffffffu, zl, bi);
-            if (nc < nnc) {
-                const uint64_t k = s_blk[s][bi];
-                const int len = (int)umin64(C::B, p.n - k * C::B);
-                const int first = lane * VPL;
-                const int cnt = first >= len ? 0 : (len - first < VPL ? len - first : VPL);
-                const uint4* slot = reinterpret_cast<const uint4*>(slot_of(s, bi)) + lane * (VPL * W / 16);
-                U u[VPL];
-#pragma unroll
-                for (int q = 0; q < VPL * W / 16; q++) reinterpret_cast<uint4*>(u)[q] = slot[q];
-                const uint32_t st = s_lc[bi][lane];
-                LaneCode lc;
-                lc.leads = st & 0xFFFFu;
-                lc.mexcl = st >> 16;
-                lc.R = s_R[bi];
-                lc.z = zb;
-                pack_block<T, VPL>(u, lc, cnt, len, stg + sb + zo);
-                if (lane == 0) zsize[nc] = (uint16_t)zb;
-            }
-        }
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&empty_bar[s]);  // this warp is done with the ring stage
-        bar_sync_named(1, C::NC);
-
-        // copy the staged tile payload to global memory with 16-byte stores
-        uint8_t* g0 = out + off_pl + excl;
-        const uintptr_t a0 = reinterpret_cast<uintptr_t>(g0), A = a0 & ~uintptr_t(15), E = a0 + agg;
-        const uint32_t nch = (uint32_t)((E - A + 15) >> 4);
-        for (uint32_t ch = threadIdx.x; ch < nch; ch += C::NC) {
-            const uintptr_t a = A + 16 * (uintptr_t)ch;
-            if (a >= a0 && a + 16 <= E) {
-                *reinterpret_cast<uint4*>(a) = *reinterpret_cast<const uint4*>(stg + 16 * ch);
+            cp_async_commit();
+        };
+        issue(0);
+        for (int b = 0; b < nbat; b++) {
+            if (b + 1 < nbat) {
+                issue(b + 1);
+                cp_async_wait<1>();
             } else {
-                for (int q = 0; q < 16; q++)
-                    if (a + q >= a0 && a + q < E) *reinterpret_cast<uint8_t*>(a + q) = stg[16 * ch + q];
+                cp_async_wait<0>();
             }
+            __syncwarp();
+            const uint32_t st = sbuf + (b & 1) * C::NB * C::BW;
+#pragma unroll 1
+            for (int j = 0; j < C::NB; j++) {
+                const int l = b * C::NB + j;
+                const uint64_t nc = g0 + l;
+                const uint32_t k = __shfl_sync(0xffffffffu, mk, l);
+                const T mu = TR::from(__shfl_sync(0xffffffffu, mmu, l));
+                const uint32_t rec = __shfl_sync(0xffffffffu, mrec, l);
+                if (nc >= c1) break;
+                T xv[VPL];
+                U uu[VPL];
+                LaneCode lc;
+                if (k < nBfull) {
+#pragma unroll
+                    for (int q = 0; q < C::QV; q++)
+                        reinterpret_cast<uint4*>(xv)[q] = lds_u128(st + j * C::BW + (lane * C::QV + q) * 16);
+                    encode_block<T, VPL>(xv, VPL, B, mu, (int)(rec & 0x7F), (rec & 0x80) != 0, eb, uu, lc);
+                } else {  // the partial tail block
+                    const int cnt = load_lane<T, VPL>(x, p.n, k, lane, xv);
+                    const int len = (int)(p.n - (uint64_t)k * B);
+                    encode_block<T, VPL>(xv, cnt, len, mu, (int)(rec & 0x7F), (rec & 0x80) != 0, eb, uu, lc);
+                }
+                if (lane == 0) {
+                    zsize[nc] = (uint16_t)lc.z;
+                    p.ncR[nc] = (uint8_t)lc.R;
+                    if (lc.R >= TR::kFull) mus[k] = 0;  // raw (NaN, Formula 4 or escalation): mu = +0 (R15)
+                }
+            }
+            __syncwarp();
+        }
+    }
+}
+
+// ------------------------------------------------------------------ K4 offsets
+// Payload offset of every write tile (kWriteTile nonconstant blocks):
+// exclusive prefix of the zsize sums, decoupled look-back over CTAs of 256
+// tiles.  The last CTA completes the header (payload bytes) and the total.
+constexpr int kWriteTile = 32;
+
+template <int W>
+__global__ void __launch_bounds__(256) k_zscan(Plan p, uint8_t* __restrict__ out) {
+    __shared__ uint64_t s_tile, s_excl, s_w[8];
+    const uint64_t nnc = *p.nnc;
+    const uint64_t ntiles = (nnc + kWriteTile - 1) / kWriteTile;
+    const uint64_t nct = (ntiles + 255) / 256;
+    if (threadIdx.x == 0) s_tile = atomicAdd(&p.ctr[2], 1u);
+    __syncthreads();
+    const uint64_t c = s_tile;
+    if (c >= nct) return;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint64_t off_zs = p.off_mu + al16((uint64_t)W * p.nB);
+    const uint16_t* zs = reinterpret_cast<const uint16_t*>(out + off_zs);
+    const uint64_t t = c * 256 + threadIdx.x;
+    uint64_t sum = 0;
+    if (t < ntiles) {
+        const uint64_t e0 = t * kWriteTile;
+        if (e0 + kWriteTile <= nnc) {
+            const uint4* q4 = reinterpret_cast<const uint4*>(zs + e0);
+#pragma unroll
+            for (int q = 0; q < kWriteTile / 8; q++) {
+                const uint4 v = q4[q];
+                sum += (v.x & 0xFFFFu) + (v.x >> 16) + (v.y & 0xFFFFu) + (v.y >> 16) + (v.z & 0xFFFFu) +
+                       (v.z >> 16) + (v.w & 0xFFFFu) + (v.w >> 16);
+            }
+        } else {
+            for (uint64_t e = e0; e < nnc; e++) sum += zs[e];
+        }
+    }
+    // CTA exclusive scan
+    uint64_t incl = sum;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint64_t v = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += v;
+    }
+    if (lane == 31) s_w[warp] = incl;
+    __syncthreads();
+    uint64_t wpre = 0, agg = 0;
+#pragma unroll
+    for (int i = 0; i < 8; i++) {
+        wpre += i < warp ? s_w[i] : 0;
+        agg += s_w[i];
+    }
+    if (warp == 0) {
+        const uint64_t e = lookback_exclusive(p.status_c, c, agg);
+        if (lane == 0) {
+            s_excl = e;
+            if (c == nct - 1) {
+                const uint64_t pbytes = e + agg;
+                p.gbase[ntiles] = pbytes;
+                reinterpret_cast<uint64_t*>(out)[6] = pbytes;  // header: payload bytes
+                *p.total = off_zs + al16(2 * nnc) + pbytes;
+            }
+        }
+    }
+    __syncthreads();
+    if (t < ntiles) p.gbase[t] = s_excl + wpre + incl - sum;
+}
+
+// ------------------------------------------------------------------ K2+K3 write pass
+// Shift / lead codes with the final R from the size pass (no guard), warp
+// scan of mid-byte counts, packing into shared memory, 16-byte stores of the
+// tile payload at its offset.  One CTA per tile, no inter-CTA dependency.
+template <typename T, int VPL>
+__device__ inline void encode_known_R(const T (&xv)[VPL], int cnt, int len, T mu, int R,
+                                      typename Traits<T>::U (&u)[VPL], LaneCode& lc) {
+    using TR = Traits<T>;
+    using U = typename TR::U;
+    const int lane = threadIdx.x & 31;
+    const bool raw = R >= TR::kFull;
+    const int s = raw ? 0 : ((8 - (R & 7)) & 7);
+    const int req = (R + s) >> 3;
+#pragma unroll
+    for (int i = 0; i < VPL; i++) u[i] = (raw ? TR::bits(xv[i]) : TR::bits(TR::sub(xv[i], mu))) >> s;
+    U prev = __shfl_up_sync(0xffffffffu, u[VPL - 1], 1);
+    if (lane == 0) prev = 0;
+    uint32_t leads = 0, m = 0;
+#pragma unroll
+    for (int i = 0; i < VPL; i++) {
+        if (i < cnt) {
+            int L = TR::clz(u[i] ^ prev) >> 3;
+            L = L > 3 ? 3 : L;
+            leads |= (uint32_t)L << (2 * i);
+            m += req > L ? req - L : 0;
+            prev = u[i];
+        }
+    }
+    const uint32_t incl = warp_incl_scan(m);
+    lc.leads = leads;
+    lc.mexcl = incl - m;
+    lc.R = R;
+    lc.z = 1 + (uint32_t)((len + 3) / 4) + __shfl_sync(0xffffffffu, incl, 31);
+}
+
+template <typename T, int VPL>
+struct WriteCfg {
+    static constexpr int W = Traits<T>::W;
+    static constexpr int B = 32 * VPL;
+    static constexpr int BW = B * W;
+    static constexpr int QV = VPL * W / 16;
+    static constexpr int TB = kWriteTile;
+    static constexpr int NWARP = 8;
+    static constexpr int BPW = TB / NWARP;
+    static constexpr int MAXZ = 1 + B / 4 + W * B;
+    static constexpr int STG = (16 + TB * MAXZ + 16 + 15) / 16 * 16;
+    static constexpr int SMEM = STG + TB * BW;   // staging + the tile's input values
+};
+
+template <typename T, int VPL>
+__global__ void __launch_bounds__(256) k_enc_write(const T* __restrict__ x, Plan p, uint8_t* __restrict__ out) {
+    using TR = Traits<T>;
+    using U = typename TR::U;
+    using C = WriteCfg<T, VPL>;
+    constexpr int W = TR::W;
+    extern __shared__ __align__(16) uint8_t stg[];
+    const uint64_t nnc = *p.nnc;
+    const uint64_t t = blockIdx.x;
+    if (t * C::TB >= nnc) return;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint64_t off_zs = p.off_mu + al16((uint64_t)W * p.nB);
+    const uint64_t off_pl = off_zs + al16(2 * nnc);
+    const uint16_t* zsize = reinterpret_cast<const uint16_t*>(out + off_zs);
+    const U* ncmu = reinterpret_cast<const U*>(p.ncmu);
+    const uint64_t nBfull = p.n / C::B;
+    // metadata of this warp's blocks (lanes 0..BPW-1), then their values via cp.async
+    const uint64_t ncw = t * C::TB + warp * C::BPW;
+    const bool mv = lane < C::BPW && ncw + lane < nnc;
+    const uint32_t mk = mv ? p.nclist[ncw + lane] : 0u;
+    const U mmu = mv ? ncmu[ncw + lane] : U(0);
+    const uint32_t mR = mv ? p.ncR[ncw + lane] : 0u;
+    const uint32_t sin = smem_u32(stg) + C::STG + warp * C::BPW * C::BW;
+#pragma unroll
+    for (int j = 0; j < C::BPW; j++) {
+        const uint32_t k = __shfl_sync(0xffffffffu, mk, j);
+        if (ncw + j < nnc && k < nBfull) {
+            const T* src = x + (uint64_t)k * C::B + lane * VPL;
+#pragma unroll
+            for (int q = 0; q < C::QV; q++) cp_async16(sin + j * C::BW + (lane * C::QV + q) * 16, src + q * (16 / W));
+        }
+    }
+    cp_async_commit();
+    // in-tile offsets of the blocks from their zsize entries
+    const uint32_t zl = t * C::TB + lane < nnc ? zsize[t * C::TB + lane] : 0u;
+    const uint32_t zincl = warp_incl_scan(zl);
+    const uint64_t base = p.gbase[t];
+    const uint32_t Tb = __shfl_sync(0xffffffffu, zincl, 31);
+    const int sb = (int)(base & 15);
+    cp_async_wait<0>();
+    __syncwarp();
+#pragma unroll 1
+    for (int j = 0; j < C::BPW; j++) {
+        const int bi = warp * C::BPW + j;
+        const uint64_t nc = t * C::TB + bi;
+        const uint32_t zo = __shfl_sync(0xffffffffu, zincl - zl, bi);
+        const uint32_t k = __shfl_sync(0xffffffffu, mk, j);
+        const T cmu = TR::from(__shfl_sync(0xffffffffu, mmu, j));
+        const int R = (int)__shfl_sync(0xffffffffu, mR, j);
+        if (nc >= nnc) break;
+        T xv[VPL];
+        U u[VPL];
+        LaneCode lc;
+        if (k < nBfull) {
+#pragma unroll
+            for (int q = 0; q < C::QV; q++)
+                reinterpret_cast<uint4*>(xv)[q] = lds_u128(sin + j * C::BW + (lane * C::QV + q) * 16);
+            encode_known_R<T, VPL>(xv, VPL, C::B, cmu, R, u, lc);
+            pack_full<T, VPL>(u, lc, smem_u32(stg) + sb + zo);
+        } else {  // the partial tail block
+            const int cnt = load_lane<T, VPL>(x, p.n, k, lane, xv);
+            const int len = (int)(p.n - (uint64_t)k * C::B);
+            encode_known_R<T, VPL>(xv, cnt, len, cmu, R, u, lc);
+            pack_block<T, VPL>(u, lc, cnt, len, stg + sb + zo);
+        }
+    }
+    __syncthreads();
+    // copy the staged tile payload to global memory with 16-byte stores
+    uint8_t* g0 = out + off_pl + base;
+    const uintptr_t a0 = reinterpret_cast<uintptr_t>(g0), A = a0 & ~uintptr_t(15), E = a0 + Tb;
+    const uint32_t nch = (uint32_t)((E - A + 15) >> 4);
+    for (uint32_t ch = threadIdx.x; ch < nch; ch += 256) {
+        const uintptr_t a = A + 16 * (uintptr_t)ch;
+        const uint4 v = *reinterpret_cast<const uint4*>(stg + 16 * ch);
+        if (a >= a0 && a + 16 <= E) {
+            *reinterpret_cast<uint4*>(a) = v;
+        } else {
+            const uint8_t* vb = reinterpret_cast<const uint8_t*>(&v);
+#pragma unroll
+            for (int q = 0; q < 16; q++)
+                if (a + q >= a0 && a + q < E) *reinterpret_cast<uint8_t*>(a + q) = vb[q];
         }
     }
 }

@@ -148,6 +148,19 @@ __device__ inline uint32_t warp_incl_scan(uint32_t v) {
     return v;
 }
 
+// ---------------------------------------------------------------- cp.async
+__device__ inline void cp_async16(uint32_t saddr, const void* g) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(saddr), "l"(g) : "memory");
+}
+__device__ inline void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ inline void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+__device__ inline uint4 lds_u128(uint32_t a) {
+    uint4 v;
+    asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
+    return v;
+}
+
 // ---------------------------------------------------------------- shared memory
 // Explicit ld.shared (generic pointers into the staging buffers otherwise
 // compile to generic LD.E).  volatile: keeps them after the mbarrier waits.
@@ -181,6 +194,43 @@ __device__ inline void run_drop4(uint32_t (&a)[NW], uint32_t k) {
 #pragma unroll
     for (int q = 0; q < NW - 1; q++) a[q] = __funnelshift_rc(a[q], a[q + 1], sh);
     a[NW - 1] = __funnelshift_rc(a[NW - 1], 0u, sh);
+}
+// Predicated shared stores (no branch, no divergence bookkeeping).
+__device__ inline void sts_u8_if(bool c, uint32_t a, uint32_t v) {
+    asm volatile("{ .reg .pred p; setp.ne.b32 p, %2, 0; @p st.shared.u8 [%0], %1; }" ::"r"(a), "r"(v), "r"((int)c)
+                 : "memory");
+}
+__device__ inline void sts_u32_if(bool c, uint32_t a, uint32_t v) {
+    asm volatile("{ .reg .pred p; setp.ne.b32 p, %2, 0; @p st.shared.u32 [%0], %1; }" ::"r"(a), "r"(v), "r"((int)c)
+                 : "memory");
+}
+// Store the first len bytes of a run (NW words) at an arbitrary shared
+// address: aligned 32-bit stores for whole words, byte stores for the
+// partial head word and the partial tail word (shared with neighbours).
+template <int NW>
+__device__ inline void run_store_s(uint32_t a, const uint32_t (&r)[NW], int len) {
+    const uint32_t base = a & ~3u;
+    const int h = (int)(a & 3u), e = h + len;
+    const uint32_t sh = 8 * (uint32_t)h;
+    uint32_t w[NW + 1];
+    w[0] = __funnelshift_lc(0u, r[0], sh);
+#pragma unroll
+    for (int q = 1; q < NW; q++) w[q] = __funnelshift_lc(r[q - 1], r[q], sh);
+    w[NW] = __funnelshift_lc(r[NW - 1], 0u, sh);
+    // whole words
+#pragma unroll
+    for (int q = 0; q <= NW; q++) sts_u32_if(4 * q >= h && 4 * q + 4 <= e, base + 4 * q, w[q]);
+    // head word (bytes h..min(4,e)-1) when it is not whole
+#pragma unroll
+    for (int j = 1; j < 4; j++) sts_u8_if(h > 0 && j >= h && j < e, base + j, w[0] >> (8 * j));
+    // tail word qt = e / 4 (bytes 0..e%4-1) unless it is word 0 with a head
+    const int qt = e >> 2;
+    uint32_t wt = w[0];
+#pragma unroll
+    for (int q = 1; q <= NW; q++) wt = q == qt ? w[q] : wt;
+    const bool tail = (e & 3) != 0 && (qt > 0 || h == 0);
+#pragma unroll
+    for (int j = 0; j < 3; j++) sts_u8_if(tail && j < (e & 3), base + 4 * qt + j, wt >> (8 * j));
 }
 // Insert k (0..4) zero bytes at the front of a run.
 template <int NW>
