@@ -62,6 +62,8 @@ def lib():
         L.orc_container_compress.restype = i64
         L.orc_container_compress.argtypes = [vp, c_int, u64, c_int, dbl, ctypes.c_uint32,
                                              ctypes.c_uint32, vp, u64]
+        L.orc_compress_shard.restype = i64
+        L.orc_compress_shard.argtypes = [vp, c_int, u64, c_int, dbl, dbl, ctypes.c_uint32, vp, u64]
         L.orc_eb_abs.restype = dbl
         L.orc_eb_abs.argtypes = [vp, c_int, u64, c_int, dbl]
         L.orc_p_f32.restype = c_int
@@ -171,6 +173,18 @@ def container_compress(x: np.ndarray, eb: float, mode: int, b: int, P: int) -> n
                                      float(eb), b, P, out.ctypes.data, cap)
     if r < 0:
         raise ValueError(f"orc_container_compress failed: {r}")
+    return out[:r].copy()
+
+
+def compress_shard(x: np.ndarray, eb_user: float, eb_abs: float, mode: int = REL, b: int = 128) -> np.ndarray:
+    """Standalone stream of a shard compressed with the GLOBAL bound eb_abs."""
+    x = np.ascontiguousarray(x).reshape(-1)
+    dt = _dtype_code(x)
+    out = np.empty(max(compress_bound(x.size, dt, b), 64), dtype=np.uint8)
+    r = lib().orc_compress_shard(x.ctypes.data if x.size else None, dt, x.size, mode, float(eb_user),
+                                 float(eb_abs), b, out.ctypes.data, out.size)
+    if r < 0:
+        raise ValueError(f"orc_compress_shard failed: {r}")
     return out[:r].copy()
 
 

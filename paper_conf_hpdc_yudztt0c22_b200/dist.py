@@ -117,7 +117,7 @@ class ShardedCompressor:
         self.rec = torch.zeros(2, dtype=torch.int64, device=device)
         ws = dist.get_world_size(group) if dist.is_available() and dist.is_initialized() else 1
         self.world = ws
-        self.records = torch.zeros(ws, 2, dtype=torch.int64, device=device)
+        self.records = torch.zeros(ws * 2, dtype=torch.int64, device=device)
 
     def compress(self, x: torch.Tensor, eb: float, mode="rel", stream=None):
         L = self._szx.lib()
@@ -139,7 +139,7 @@ class ShardedCompressor:
         if self.world > 1:
             dist.all_gather_into_tensor(self.records, self.rec, group=self.group)
         else:
-            self.records[0].copy_(self.rec)
+            self.records.copy_(self.rec)
 
     def stream(self) -> torch.Tensor:
         """This rank's stream (synchronises to read its length)."""
@@ -147,24 +147,40 @@ class ShardedCompressor:
 
     def container_offsets(self):
         """(firsts, offsets, total container bytes) from the all-gathered records (host sync)."""
-        r = self.records.cpu().tolist()
+        r = self.records.view(-1, 2).cpu().tolist()
         return container_layout([int(a) for a, _ in r], [int(bb) for _, bb in r])
 
 
-def gather_container(sc: ShardedCompressor, dst: int = 0, group=None) -> torch.Tensor | None:
-    """Collect every rank's stream on rank dst and build the SZXC container there."""
-    s = sc.stream()
-    r = sc.records.cpu().tolist()
+def allgather_records(n_elem: int, nbytes: torch.Tensor, group=None) -> torch.Tensor:
+    """All-gather of each rank's (n_elem, stream bytes) record -> [P, 2] int64 (same device)."""
+    rec = torch.stack([torch.full_like(nbytes.view(-1)[:1], n_elem).view(()), nbytes.view(-1)[0]]).to(torch.int64)
+    if not (dist.is_available() and dist.is_initialized()) or dist.get_world_size(group) == 1:
+        return rec.view(1, 2)
+    out = torch.empty(dist.get_world_size(group) * 2, dtype=torch.int64, device=rec.device)
+    dist.all_gather_into_tensor(out, rec.contiguous(), group=group)
+    return out.view(-1, 2)
+
+
+def gather_streams(stream: torch.Tensor, records: torch.Tensor, dst: int = 0, group=None) -> torch.Tensor | None:
+    """Collect every rank's stream on rank dst and build the SZXC container there
+    (records = allgather_records output).  Works for NCCL (CUDA) and gloo (CPU)."""
+    r = records.cpu().tolist()
     n_elems = [int(a) for a, _ in r]
     nbytes = [int(bb) for _, bb in r]
-    if sc.world == 1:
-        return build_container([s], n_elems)
+    world = len(r)
+    if world == 1:
+        return build_container([stream], n_elems)
     mx = max(nbytes)
-    pad = torch.zeros(mx, dtype=torch.uint8, device=s.device)
-    pad[: s.numel()] = s
+    pad = torch.zeros(mx, dtype=torch.uint8, device=stream.device)
+    pad[: stream.numel()] = stream
     rank = dist.get_rank(group)
-    bufs = [torch.empty(mx, dtype=torch.uint8, device=s.device) for _ in range(sc.world)] if rank == dst else None
+    bufs = [torch.empty(mx, dtype=torch.uint8, device=stream.device) for _ in range(world)] if rank == dst else None
     dist.gather(pad, bufs, dst=dst, group=group)
     if rank != dst:
         return None
     return build_container([b[:nb] for b, nb in zip(bufs, nbytes)], n_elems)
+
+
+def gather_container(sc: ShardedCompressor, dst: int = 0, group=None) -> torch.Tensor | None:
+    """Collect every rank's stream on rank dst and build the SZXC container there."""
+    return gather_streams(sc.stream(), sc.records.view(-1, 2), dst, group)

@@ -9,4 +9,4 @@ timeout ${TEST_TIMEOUT:-1200} python -m pytest tests -m gpu -x -q ${PYTEST_ARGS}
 if [ -z "$NO_BENCH" ]; then
 timeout 600 python bench.py ${BENCH_ARGS} > gpurun_out/bench.log 2>&1; echo "bench rc=$?" >> gpurun_out/bench.log
 fi
-tail -3 gpurun_out/smoke.log; tail -15 gpurun_out/pytest_gpu.log; tail -c 3000 gpurun_out/bench.log
+tail -3 gpurun_out/smoke.log; tail -15 gpurun_out/pytest_gpu.log; [ -f gpurun_out/bench.log ] && tail -c 3000 gpurun_out/bench.log; true
