@@ -113,6 +113,20 @@ def _cpu_info():
     return model, os.cpu_count()
 
 
+def _ncu_traffic(kernel: str):
+    """dram__bytes_read.sum + dram__bytes_write.sum of `kernel` (one launch) from the newest
+    committed ncu --set full summary under profiles/, or None."""
+    import glob
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "r*_ncu_full_summary.json")))
+    if not files:
+        return None, None
+    d = json.load(open(files[-1]))
+    for name, v in d.items():
+        if name.startswith(kernel + "<") or name == kernel:
+            return v.get("dram_bytes"), os.path.basename(files[-1])
+    return None, None
+
+
 def _peaks():
     try:
         return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"], "measured"
@@ -300,8 +314,10 @@ def main():
         nB = (n_el + 127) // 128
         alg = {
             "k_block_stats": nbytes + nB * 8,
-            "k_classify": nB * 8 + nB * 4 + nB // 8,
-            "k_encode": nnc * 128 * 4 + nB * 8 + 2 * nnc + pb,
+            "k_classify": nB * 8 + nB * 4 + nB // 8 + 9 * nnc,
+            "k_enc_size": nnc * 128 * 4 + 2 * nnc + 5 * nnc,
+            "k_zscan": 2 * nnc,
+            "k_enc_write": nnc * 128 * 4 + 5 * nnc + pb,
             "k_index": nB // 8 + 2 * nnc,
             "k_decode": S + nbytes,
         }
@@ -309,8 +325,9 @@ def main():
         roof = None
         if dom:
             ach = alg.get(dom, 0) / (kms[dom] / 1e3) / 1e9
+            traffic, src = _ncu_traffic(dom)
             roof = {"kernel": dom, "bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s",
-                    "frac": ach / peak, "peak_kind": peak_kind, "traffic": None,
+                    "frac": ach / peak, "peak_kind": peak_kind, "traffic": traffic, "traffic_source": src,
                     "alg_bytes_per_launch": alg.get(dom), "ms_per_launch": kms[dom]}
         comp_alg = 2 * nbytes + S   # REL: range pass + encode
         dec_alg = S + nbytes
