@@ -299,7 +299,7 @@ __device__ inline bool decode_full(uint32_t src, uint32_t z, T mu, T (&out)[VPL]
         const int mi = req > L ? req - L : 0;
         U bytes;
         if (W == 4) {
-            bytes = run[0] & (mi >= 4 ? 0xFFFFFFFFu : ((1u << (8 * mi)) - 1u));
+            bytes = run[0] & ~__funnelshift_lc(0u, 0xFFFFFFFFu, 8 * mi);  // low mi bytes (mi = 4: all)
             run_drop4<NW>(run, mi);
         } else {
             bytes = ((U)run[0] | ((U)run[1] << 16 << 16)) & (mi >= 8 ? ~U(0) : ((U(1) << (8 * mi)) - U(1)));
@@ -308,7 +308,7 @@ __device__ inline bool decode_full(uint32_t src, uint32_t z, T mu, T (&out)[VPL]
         }
         own[i] = bytes << (8 * (W - req));
         const int copy = L < req ? L : req;  // (2) bytes copied from the previous value
-        cmk[i] = copy == 0 ? U(0) : (~U(0) << (8 * (W - copy)));
+        cmk[i] = ~(~U(0) >> (8 * copy));     // top `copy` bytes (copy <= 3 < W)
         M &= cmk[i];
         D = (D & cmk[i]) | own[i];
     }
@@ -430,51 +430,66 @@ __global__ void __launch_bounds__(DecodeCfg<T, VPL>::NT, DecodeCfg<T, VPL>::MINB
     }
 
     // ---------------- consumers
+    const uint32_t sbase = smem_u32(smem);
+    const uint64_t nW_full = p.n / ((uint64_t)C::TB * C::B);   // tiles whose 32 blocks are all full
+    constexpr int NV = VPL * C::W / 16;                          // 16-byte stores per lane per block
+    constexpr int QB = C::B * C::W / 16;                         // 16-byte chunks per block
+    const uint32_t below = (1u << lane) - 1u;
     int i = 0;
     for (uint64_t t = blockIdx.x; t < p.nW; t += G, i++) {
         const int s = i % C::STAGES;
         mbar_wait(&full_bar[s], (i / C::STAGES) & 1);
-        const uint8_t* pay = smem + (size_t)s * C::STAGE;
-        const U* mub = reinterpret_cast<const U*>(pay + C::PAY);
+        const uint32_t pay = sbase + s * C::STAGE;
+        const uint32_t mub = pay + C::PAY;
         const uint32_t word = s_word[s];
         const uint32_t cnt = __popc(word);
+        // zsize of the tile's nonconstant blocks (lane r holds the r-th); validate once
         const uint32_t zl = (s_ok[s] && (uint32_t)lane < cnt) ? s_zw[s][s_zo[s] + lane] : 0u;
-        const uint32_t zincl = warp_incl_scan(zl);
-        const uint32_t zoff = zincl - zl;  // offset of the lane-th nonconstant block
         const bool zok = (uint32_t)lane >= cnt || (zl >= 2 && zl <= (uint32_t)C::MAXZ);
-        const bool ok = s_ok[s] && __all_sync(0xffffffffu, zok) && __shfl_sync(0xffffffffu, zincl, 31) == s_T[s];
+        const bool ok = s_ok[s] && __all_sync(0xffffffffu, zok) && __reduce_add_sync(0xffffffffu, zl) == s_T[s];
+        const uint32_t mine = (word >> (warp * C::BPW)) & ((1u << C::BPW) - 1u);  // my nonconstant blocks
         if (!ok) {
             if (threadIdx.x == 0) set_corrupt(p.err);
-        } else if ((t + 1) * C::TB * C::B <= p.n) {
+        } else if (t < nW_full) {
             // full tile: every block holds B values
-            const uint32_t spay = smem_u32(pay) + s_sb[s];
-            const uint32_t smu = smem_u32(mub) + warp * C::BPW * C::W;
+            const uint32_t spay = pay + s_sb[s];
+            const uint32_t smu = mub + warp * C::BPW * C::W;
             uint4* yq = reinterpret_cast<uint4*>(y + (t * C::TB + warp * C::BPW) * C::B + lane * VPL);
-            constexpr int NV = VPL * C::W / 16;       // 16-byte stores per lane per block
-            constexpr int QB = C::B * C::W / 16;      // 16-byte chunks per block
-#pragma unroll 1
+            // constant blocks: retrieve with mu (Fig. 10, state 0)
+#pragma unroll
             for (int j = 0; j < C::BPW; j++) {
+                if (!((mine >> j) & 1u)) {
+                    U mb = lds_u32(smu + j * C::W);
+                    if (C::W == 8) mb |= (U)lds_u32(smu + j * C::W + 4) << 16 << 16;
+                    T v[VPL];
+#pragma unroll
+                    for (int q = 0; q < VPL; q++) v[q] = TR::from(mb);
+#pragma unroll
+                    for (int q = 0; q < NV; q++) yq[j * QB + q] = reinterpret_cast<const uint4*>(v)[q];
+                }
+            }
+            // nonconstant blocks
+#pragma unroll 1
+            for (uint32_t m = mine; m; m &= m - 1) {
+                const int j = __ffs(m) - 1;
                 const int idx = warp * C::BPW + j;
+                const uint32_t rank = __popc(word & ((1u << idx) - 1u));
+                const uint32_t off = __reduce_add_sync(0xffffffffu, (uint32_t)lane < rank ? zl : 0u);
+                const uint32_t z = __shfl_sync(0xffffffffu, zl, rank);
                 U mb = lds_u32(smu + j * C::W);
                 if (C::W == 8) mb |= (U)lds_u32(smu + j * C::W + 4) << 16 << 16;
-                const T mu = TR::from(mb);
                 T v[VPL];
-                if (!((word >> idx) & 1u)) {
-#pragma unroll
-                    for (int q = 0; q < VPL; q++) v[q] = mu;  // constant block: retrieve with mu
-                } else {
-                    const uint32_t rank = __popc(word & ((1u << idx) - 1u));
-                    const uint32_t off = __shfl_sync(0xffffffffu, zoff, rank);
-                    const uint32_t z = __shfl_sync(0xffffffffu, zl, rank);
-                    if (!decode_full<T, VPL>(spay + off, z, mu, v)) {
-                        if (lane == 0) set_corrupt(p.err);
-                        continue;
-                    }
+                if (!decode_full<T, VPL>(spay + off, z, TR::from(mb), v)) {
+                    if (lane == 0) set_corrupt(p.err);
+                    continue;
                 }
 #pragma unroll
                 for (int q = 0; q < NV; q++) yq[j * QB + q] = reinterpret_cast<const uint4*>(v)[q];
             }
         } else {
+            // last (partial) tile: generic path with bounds and tail handling
+            const uint8_t* gpay = smem + (size_t)s * C::STAGE;
+            const U* gmu = reinterpret_cast<const U*>(gpay + C::PAY);
             const int sb = (int)s_sb[s];
 #pragma unroll 1
             for (int j = 0; j < C::BPW; j++) {
@@ -482,16 +497,16 @@ __global__ void __launch_bounds__(DecodeCfg<T, VPL>::NT, DecodeCfg<T, VPL>::MINB
                 const uint64_t k = t * C::TB + idx;
                 if (k >= p.nB) break;
                 const int len = (int)umin64(C::B, p.n - k * C::B);
-                const T mu = TR::from(mub[idx]);
+                const T mu = TR::from(gmu[idx]);
                 T v[VPL];
                 if (!((word >> idx) & 1u)) {
 #pragma unroll
-                    for (int q = 0; q < VPL; q++) v[q] = mu;  // constant block: retrieve with mu
+                    for (int q = 0; q < VPL; q++) v[q] = mu;
                 } else {
                     const uint32_t rank = __popc(word & ((1u << idx) - 1u));
-                    const uint32_t off = __shfl_sync(0xffffffffu, zoff, rank);
+                    const uint32_t off = __reduce_add_sync(0xffffffffu, (uint32_t)lane < rank ? zl : 0u);
                     const uint32_t z = __shfl_sync(0xffffffffu, zl, rank);
-                    if (!decode_block<T, VPL>(pay + sb + off, z, len, mu, v)) {
+                    if (!decode_block<T, VPL>(gpay + sb + off, z, len, mu, v)) {
                         if (lane == 0) set_corrupt(p.err);
                         continue;
                     }
@@ -499,6 +514,7 @@ __global__ void __launch_bounds__(DecodeCfg<T, VPL>::NT, DecodeCfg<T, VPL>::MINB
                 store_lane<T, VPL>(y, p.n, k, lane, v);
             }
         }
+        (void)below;
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty_bar[s]);
     }
