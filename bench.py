@@ -247,8 +247,8 @@ def main():
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    szx.timing_reset()
-    szx.timing_enable(True)
+    # ---- timed region (the contract's K steps): kernels chained with programmatic
+    # dependent launch, per-phase events only (between compress and decompress)
     l0 = szx.launch_count()
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True),
             torch.cuda.Event(enable_timing=True)) for _ in range(a.steps)]
@@ -269,8 +269,6 @@ def main():
         dist.barrier()
     torch.cuda.synchronize()
     launches = szx.launch_count() - l0
-    szx.timing_enable(False)
-    kt = szx.timing_read()
     total_ms = e_start.elapsed_time(e_end)
     comp_ms = statistics.median([e0.elapsed_time(e1) for e0, e1, _ in evs])
     dec_ms = statistics.median([e1.elapsed_time(e2) for _, e1, e2 in evs])
@@ -279,6 +277,15 @@ def main():
         t = torch.tensor([ms_step, comp_ms, dec_ms], device=dev, dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms_step, comp_ms, dec_ms = t.tolist()
+    # ---- per-kernel pass: the library records CUDA events around every launch on
+    # its launch stream (this serialises the launches, so it is a separate pass)
+    szx.timing_reset()
+    szx.timing_enable(True)
+    for i in range(min(a.steps, 100)):
+        step()
+    torch.cuda.synchronize()
+    szx.timing_enable(False)
+    kt = szx.timing_read()
     clocks = sampler.summary(t_wall0, t_wall1) if sampler else None
 
     # ---------------- end to end through the C ABI host entry points (pinned host buffers)
@@ -348,6 +355,9 @@ def main():
             "max_abs_err": err, "eb_abs": hdr.eb_abs,
             "roofline": roof, "kernels_ms_per_launch": kms, "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": launches, "clocks": clocks,
+            "timing": "value/ms_per_step: CUDA events around the K timed steps (kernels chained with PDL); "
+                      "kernels_ms_per_launch/roofline: library CUDA events around each launch in a second "
+                      "pass of min(K,100) steps",
             "paper_context": "cuSZx A100: 150-216 GB/s compress, 150-291 GB/s decompress (P:L3207-3220)",
         }
         print(json.dumps(out), flush=True)

@@ -70,6 +70,28 @@ void launch(const char* name, cudaStream_t s, F&& f) {
     g_launches++;
 }
 
+std::atomic<bool> g_timing_on{false};  // mirrors Timing::on without taking its mutex
+bool timing_on() { return g_timing_on.load(); }
+
+// cudaLaunchKernelEx with programmatic stream serialization (PDL): the kernel
+// may start launching while its predecessor drains; it calls pdl_wait() before
+// touching the predecessor's output.  Disabled while per-kernel timing events
+// sit between the launches.
+template <typename... KArgs, typename... Args>
+void launch_pdl(void (*k)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s, Args... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = timing_on() ? 0 : 1;
+    cudaLaunchKernelEx(&cfg, k, static_cast<KArgs>(args)...);
+}
+
 void timing_resolve() {
     Timing& T = timing();
     std::lock_guard<std::mutex> g(T.mu);
@@ -193,7 +215,7 @@ void enqueue_stats(const void* d_in, const Plan& p, int want_range, cudaStream_t
 template <typename T, int VPL>
 void enqueue_encode(const void* d_in, const Plan& p, const CLayout& L, uint8_t* out, cudaStream_t s) {
     set_smem_attrs<T, VPL>();
-    launch("k_classify", s, [&] { k_classify<T><<<(unsigned)L.nTB, 256, 0, s>>>(p, out); });
+    launch("k_classify", s, [&] { launch_pdl(k_classify<T>, dim3((unsigned)L.nTB), dim3(256), 0, s, p, out); });
     static int occ = 0;
     if (!occ) {
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_enc_size<T, VPL>, 256, SizeCfg<T, VPL>::SMEM);
@@ -204,13 +226,14 @@ void enqueue_encode(const void* d_in, const Plan& p, const CLayout& L, uint8_t* 
     if (grid > cap) grid = cap;
     if (grid == 0) grid = 1;
     launch("k_enc_size", s, [&] {
-        k_enc_size<T, VPL><<<(unsigned)grid, 256, SizeCfg<T, VPL>::SMEM, s>>>(static_cast<const T*>(d_in), p, out);
+        launch_pdl(k_enc_size<T, VPL>, dim3((unsigned)grid), dim3(256), SizeCfg<T, VPL>::SMEM, s,
+                   static_cast<const T*>(d_in), p, out);
     });
-    launch("k_zscan", s, [&] { k_zscan<Traits<T>::W><<<(unsigned)L.nTC, 256, 0, s>>>(p, out); });
+    launch("k_zscan", s, [&] { launch_pdl(k_zscan<Traits<T>::W>, dim3((unsigned)L.nTC), dim3(256), 0, s, p, out); });
     using C = WriteCfg<T, VPL>;
     launch("k_enc_write", s, [&] {
-        k_enc_write<T, VPL><<<(unsigned)cdiv(L.nB, kWriteTile), 256, C::SMEM, s>>>(static_cast<const T*>(d_in), p,
-                                                                                   out);
+        launch_pdl(k_enc_write<T, VPL>, dim3((unsigned)cdiv(L.nB, kWriteTile)), dim3(256), C::SMEM, s,
+                   static_cast<const T*>(d_in), p, out);
     });
 }
 
@@ -220,7 +243,7 @@ void dispatch(szx_dtype_t dt, uint32_t b, F&& f);
 // Enqueue the whole compression.  Returns SZX_OK or an error.
 int enqueue_compress(const void* d_in, szx_dtype_t dt, uint64_t n, szx_ebmode_t mode, double eb,
                      uint32_t b, void* d_out, uint64_t cap, void* d_ws, uint64_t ws_bytes,
-                     uint64_t** d_total_out, cudaStream_t s) {
+                     uint64_t** d_total_out, cudaStream_t s, uint64_t* user_total = nullptr) {
     int rc = check_compress_args(d_in, dt, n, mode, eb, b, d_out);
     if (rc) return rc;
     if (!have_device()) return SZX_ECUDA;
@@ -232,6 +255,7 @@ int enqueue_compress(const void* d_in, szx_dtype_t dt, uint64_t n, szx_ebmode_t 
     uint8_t* ws = static_cast<uint8_t*>(d_ws);
     uint8_t* out = static_cast<uint8_t*>(d_out);
     Plan p = make_plan(L, ws, n, dt, mode, eb, b, nullptr);
+    if (user_total) p.total = user_total;  // the kernels write the stream length straight there
     *d_total_out = p.total;
     if (n == 0) {
         launch("k_empty_header", s, [&] { k_empty_header<<<1, 1, 0, s>>>(out, dt, mode, b, eb, nullptr, p.total); });
@@ -356,7 +380,7 @@ int enqueue_decompress(const void* d_in, uint64_t in_bytes, const szx_header_t* 
         const uint64_t cap = (uint64_t)sm_count() * occ;
         if (grid > cap) grid = cap;
         launch("k_decode", s, [&] {
-            k_decode<T, V><<<(unsigned)grid, C::NT, C::SMEM, s>>>(p, in, static_cast<T*>(d_out));
+            launch_pdl(k_decode<T, V>, dim3((unsigned)grid), dim3(C::NT), C::SMEM, s, p, in, static_cast<T*>(d_out));
         });
     });
     return cudaGetLastError() == cudaSuccess ? SZX_OK : SZX_ECUDA;
@@ -406,11 +430,7 @@ int szx_compress_async(const void* d_in, szx_dtype_t dt, uint64_t n, szx_ebmode_
                        uint64_t* d_total_bytes, void* stream) {
     cudaStream_t s = static_cast<cudaStream_t>(stream);
     uint64_t* d_tot = nullptr;
-    int rc = enqueue_compress(d_in, dt, n, mode, eb, b, d_out, cap, d_ws, ws_bytes, &d_tot, s);
-    if (rc) return rc;
-    if (d_total_bytes && d_total_bytes != d_tot)
-        if (cudaMemcpyAsync(d_total_bytes, d_tot, 8, cudaMemcpyDeviceToDevice, s) != cudaSuccess) return SZX_ECUDA;
-    return SZX_OK;
+    return enqueue_compress(d_in, dt, n, mode, eb, b, d_out, cap, d_ws, ws_bytes, &d_tot, s, d_total_bytes);
 }
 
 int64_t szx_compress_ws(const void* d_in, szx_dtype_t dt, uint64_t n, szx_ebmode_t mode, double eb,
@@ -631,6 +651,7 @@ void szx_timing_enable(int on) {
     Timing& T = timing();
     std::lock_guard<std::mutex> g(T.mu);
     T.on = on != 0;
+    g_timing_on.store(on != 0);
 }
 void szx_timing_reset(void) {
     Timing& T = timing();

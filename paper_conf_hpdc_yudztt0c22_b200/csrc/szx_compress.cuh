@@ -259,6 +259,8 @@ __global__ void __launch_bounds__(256) k_classify(Plan p, uint8_t* __restrict__ 
     using U = typename TR::U;
     __shared__ uint64_t s_tile, s_base;
     __shared__ uint32_t s_cnt[64], s_pre[64];
+    pdl_wait();
+    pdl_trigger();
     if (threadIdx.x == 0) s_tile = atomicAdd(&p.ctr[0], 1u);
     __syncthreads();
     const uint64_t tile = s_tile;
@@ -525,6 +527,8 @@ __global__ void __launch_bounds__(256) k_enc_size(const T* __restrict__ x, Plan 
     constexpr int B = C::B;
     extern __shared__ __align__(16) uint8_t smem[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    pdl_wait();
+    pdl_trigger();
     const uint64_t nnc = *p.nnc;
     const double eb = *p.eb_abs;
     const uint64_t off_zs = p.off_mu + al16((uint64_t)W * p.nB);
@@ -611,6 +615,8 @@ constexpr int kWriteTile = 32;
 template <int W>
 __global__ void __launch_bounds__(256) k_zscan(Plan p, uint8_t* __restrict__ out) {
     __shared__ uint64_t s_tile, s_excl, s_w[8];
+    pdl_wait();
+    pdl_trigger();
     const uint64_t nnc = *p.nnc;
     const uint64_t ntiles = (nnc + kWriteTile - 1) / kWriteTile;
     const uint64_t nct = (ntiles + 255) / 256;
@@ -724,6 +730,8 @@ __global__ void __launch_bounds__(256) k_enc_write(const T* __restrict__ x, Plan
     using C = WriteCfg<T, VPL>;
     constexpr int W = TR::W;
     extern __shared__ __align__(16) uint8_t stg[];
+    pdl_wait();
+    pdl_trigger();
     const uint64_t nnc = *p.nnc;
     const uint64_t t = blockIdx.x;
     if (t * C::TB >= nnc) return;

@@ -345,6 +345,8 @@ __global__ void __launch_bounds__(DecodeCfg<T, VPL>::NT, DecodeCfg<T, VPL>::MINB
     __shared__ uint32_t s_word[C::STAGES], s_sb[C::STAGES], s_zo[C::STAGES], s_ok[C::STAGES];
     __shared__ uint64_t s_T[C::STAGES];
 
+    pdl_wait();
+    pdl_trigger();
     const DHdr hd = read_dheader<TR::W>(in, p);
     if (!hd.ok) return;  // k_index has flagged it
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;

@@ -148,6 +148,13 @@ __device__ inline uint32_t warp_incl_scan(uint32_t v) {
     return v;
 }
 
+// ---------------------------------------------------------------- PDL
+// Programmatic dependent launch: wait until the preceding kernel in the stream
+// has completed and its memory is visible (no-op when launched without PDL),
+// and let the next kernel start launching while this one drains.
+__device__ inline void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ inline void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
 // ---------------------------------------------------------------- cp.async
 __device__ inline void cp_async16(uint32_t saddr, const void* g) {
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(saddr), "l"(g) : "memory");
