@@ -186,7 +186,7 @@ void set_smem_attrs() {
     if (done) return;
     cudaFuncSetAttribute(k_enc_write<T, VPL>, cudaFuncAttributeMaxDynamicSharedMemorySize, WriteCfg<T, VPL>::SMEM);
     cudaFuncSetAttribute(k_enc_size<T, VPL>, cudaFuncAttributeMaxDynamicSharedMemorySize, SizeCfg<T, VPL>::SMEM);
-    cudaFuncSetAttribute(k_decode<T, VPL>, cudaFuncAttributeMaxDynamicSharedMemorySize, DecodeCfg<T, VPL>::SMEM);
+
     done = true;
 }
 
@@ -368,19 +368,19 @@ int enqueue_decompress(const void* d_in, uint64_t in_bytes, const szx_header_t* 
     dispatch((szx_dtype_t)h->dtype, h->block_size, [&](auto tag, auto vpl) {
         using T = decltype(tag);
         constexpr int V = decltype(vpl)::value;
-        set_smem_attrs<T, V>();
-        using C = DecodeCfg<T, V>;
         launch("k_index", s, [&] { k_index<Traits<T>::W><<<(unsigned)L.nTI, 256, 0, s>>>(p, in); });
+        // one warp per 32-block tile, grid-stride; enough CTAs for full occupancy
         static int occ = 0;
         if (!occ) {
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_decode<T, V>, C::NT, C::SMEM);
-            if (occ <= 0) occ = 1;
+            cudaFuncSetAttribute(k_decode_w<T, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, DecWCfg<T, V>::SMEM);
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_decode_w<T, V>, 256, DecWCfg<T, V>::SMEM);
+            if (occ <= 0) occ = 4;
         }
-        uint64_t grid = L.nW;
+        uint64_t grid = cdiv(L.nW, 8);
         const uint64_t cap = (uint64_t)sm_count() * occ;
         if (grid > cap) grid = cap;
         launch("k_decode", s, [&] {
-            launch_pdl(k_decode<T, V>, dim3((unsigned)grid), dim3(C::NT), C::SMEM, s, p, in, static_cast<T*>(d_out));
+            launch_pdl(k_decode_w<T, V>, dim3((unsigned)grid), dim3(256), DecWCfg<T, V>::SMEM, s, p, in, static_cast<T*>(d_out));
         });
     });
     return cudaGetLastError() == cudaSuccess ? SZX_OK : SZX_ECUDA;

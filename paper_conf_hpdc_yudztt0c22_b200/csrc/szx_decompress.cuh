@@ -8,12 +8,11 @@
 //               (b) payload byte offset of each tile = prefix of its zsize
 //                   sums (the CTA's zsize range is staged in shared memory).
 //             Totals are validated against the header (nNC, payload size).
-//   k_decode  (K5)  persistent and warp-specialised: a producer warp reads a
-//             tile's metadata and issues ONE TMA bulk copy of the tile's
-//             contiguous payload (plus one for its 32 mu values) into a
-//             shared-memory ring; 8 consumer warps rebuild the values with
-//             the five steps of Fig. 10 and write them with
-//             16-byte stores.  The leading-byte dependence chains
+//   k_decode_w (K5) a warp per 32-block tile (grid-stride): metadata, mu
+//             values, zsize entries and the nonconstant payloads are read
+//             straight from global memory; the values are rebuilt with the
+//             five steps of Fig. 10 and written with 16-byte
+//             stores.  The leading-byte dependence chains
 //             (Challenge 2) are resolved with a warp scan of
 //             byte-mask transfer functions instead of the paper's log-step
 //             index propagation: a lane's values map an
@@ -31,7 +30,7 @@ struct DPlan {
     uint64_t n, nB, nW, in_bytes;
     uint64_t off_mu;
     uint32_t b, dtype;
-    uint32_t* ctr;             // [2] tickets, init 0
+    uint32_t* ctr;             // [2] init 0: k_index tile ticket, k_decode_w tile counter
     uint64_t* status_a;        // init 0
     uint64_t* status_z;        // init 0
     uint32_t* ncpre;           // [nW]      nonconstant index of each tile's first block
@@ -144,23 +143,6 @@ __global__ void __launch_bounds__(256) k_index(DPlan p, const uint8_t* __restric
 }
 
 template <typename T, int VPL>
-struct DecodeCfg {
-    static constexpr int W = Traits<T>::W;
-    static constexpr int B = 32 * VPL;
-    static constexpr int TB = kTileBlocks;                 // blocks per tile (one bitmap word)
-    static constexpr int NWARP = 8;                        // consumer warps
-    static constexpr int BPW = TB / NWARP;
-    static constexpr int NT = (NWARP + 1) * 32;            // + producer warp
-    static constexpr int MAXZ = 1 + B / 4 + W * B;
-    static constexpr int PAY = (TB * MAXZ + 32 + 15) / 16 * 16;  // + up to 15 lead / trail bytes
-    static constexpr int MUB = TB * W;
-    static constexpr int STAGE = PAY + MUB;
-    static constexpr int STAGES = (W == 4 && VPL == 4) ? 3 : 2;
-    static constexpr int SMEM = STAGES * STAGE;
-    static constexpr int MINB = (W == 4 && VPL == 4) ? 3 : 2;
-};
-
-template <typename T, int VPL>
 __device__ inline void store_lane(T* __restrict__ y, uint64_t n, uint64_t k, int lane, const T (&v)[VPL]) {
     constexpr int B = 32 * VPL;
     const uint64_t first = k * B + (uint64_t)lane * VPL;
@@ -176,15 +158,56 @@ __device__ inline void store_lane(T* __restrict__ y, uint64_t n, uint64_t k, int
         if (first + i < n) y[first + i] = v[i];
 }
 
-// Decode one nonconstant block whose payload (z bytes) starts at src (smem).
-template <typename T, int VPL>
-__device__ inline bool decode_block(const uint8_t* src, uint32_t z, int len, T mu, T (&out)[VPL]) {
+namespace gsrc {
+// generic-address loads: the source is either a shared-memory staging slot or
+// the stream in global memory (fallback for oversized tiles)
+__device__ inline uint32_t ldg_u8(const uint8_t* p) { return *p; }
+__device__ inline uint32_t ldg_u32(const void* p) { return *reinterpret_cast<const uint32_t*>(p); }
+// run of bytes at an arbitrary address, realigned; aligned words that start at
+// or past `lim` (one past the last valid byte) read as 0.  An aligned word
+// holding at least one stream byte never leaves the (>=16-B aligned) buffer.
+template <int NW>
+__device__ inline void run_load(const uint8_t* p, uintptr_t lim4, uint32_t (&r)[NW]) {
+    const uintptr_t a = reinterpret_cast<uintptr_t>(p);
+    const uintptr_t base = a & ~uintptr_t(3);
+    const uint32_t sh = 8 * (uint32_t)(a & 3);
+    uint32_t lo = base < lim4 ? ldg_u32(reinterpret_cast<const void*>(base)) : 0u;
+#pragma unroll
+    for (int q = 0; q < NW; q++) {
+        const uintptr_t aq = base + 4 * (q + 1);
+        const uint32_t hi = aq < lim4 ? ldg_u32(reinterpret_cast<const void*>(aq)) : 0u;
+        r[q] = __funnelshift_r(lo, hi, sh);
+        lo = hi;
+    }
+}
+}  // namespace gsrc
+
+// Where a nonconstant block's payload is read from: the stream in global
+// memory (bounded by the end of the buffer) or a shared-memory staging slot.
+struct SrcG {
+    const uint8_t* p;
+    uintptr_t lim;
+    __device__ uint32_t u8(uint32_t o) const { return gsrc::ldg_u8(p + o); }
+    template <int NW>
+    __device__ void run(uint32_t o, uint32_t (&r)[NW]) const { gsrc::run_load<NW>(p + o, lim, r); }
+};
+struct SrcS {
+    uint32_t a;  // shared-window address
+    __device__ uint32_t u8(uint32_t o) const { return lds_u8(a + o); }
+    template <int NW>
+    __device__ void run(uint32_t o, uint32_t (&r)[NW]) const { run_load_s<NW>(a + o, r); }
+};
+
+// Decode one nonconstant block (any length) whose payload (z bytes) starts at src (global).
+template <typename T, int VPL, typename Src>
+__device__ inline bool decode_block_g(const Src src, uint32_t z, int len, T mu,
+                                      T (&out)[VPL]) {
     using TR = Traits<T>;
     using U = typename TR::U;
     constexpr int W = TR::W;
     const int lane = threadIdx.x & 31;
     const int ncode = (len + 3) / 4;
-    const int R = src[0];
+    const int R = (int)src.u8(0);
     if (R < TR::kFloor || R > TR::kFull) return false;
     const bool raw = R >= TR::kFull;
     const int s = raw ? 0 : ((8 - (R & 7)) & 7);
@@ -196,7 +219,7 @@ __device__ inline bool decode_block(const uint8_t* src, uint32_t z, int len, T m
 #pragma unroll
     for (int q = 0; q < VPL / 4; q++) {
         const int cb = lane * (VPL / 4) + q;
-        if (cb < ncode) leads |= (uint32_t)src[1 + cb] << (8 * q);
+        if (cb < ncode) leads |= src.u8(1 + cb) << (8 * q);
     }
     uint32_t m = 0;
 #pragma unroll
@@ -212,7 +235,7 @@ __device__ inline bool decode_block(const uint8_t* src, uint32_t z, int len, T m
     // funnel shifts; value i takes the next m_i bytes of the run.
     constexpr int NW = VPL * W / 4;
     uint32_t run[NW];
-    run_load<NW>(src + 1 + ncode + (incl - m), run);
+    src.template run<NW>(1 + ncode + (incl - m), run);
     U own[VPL];
     U M = ~U(0), D = 0;  // lane map: c -> (c & M) | D
 #pragma unroll
@@ -260,26 +283,32 @@ __device__ inline bool decode_block(const uint8_t* src, uint32_t z, int len, T m
     return true;
 }
 
-// Fast path of decode_block for a FULL block (every lane holds VPL values):
-// no per-value tail guards, explicit ld.shared, clamped funnel shifts.
-// src is the shared-memory address of the block payload.
-template <typename T, int VPL>
-__device__ inline bool decode_full(uint32_t src, uint32_t z, T mu, T (&out)[VPL]) {
+// ===================================================================== K5w
+// Warp-granular decoder: a warp owns whole 32-block tiles (grid-stride), reads
+// the tile's metadata, mu values, zsize entries and the nonconstant payloads
+// straight from global memory (read-only path), and writes 16-byte stores.
+// No shared-memory ring, no block-level barriers: latency is hidden by having
+// many independent warps per SM, and the per-tile bookkeeping is amortised
+// over 32 blocks per warp.
+
+
+// decode_full with the payload in global memory
+template <typename T, int VPL, typename Src>
+__device__ inline bool decode_full_g(const Src src, uint32_t z, T mu, T (&out)[VPL]) {
     using TR = Traits<T>;
     using U = typename TR::U;
     constexpr int W = TR::W;
-    constexpr int NCODE = 8 * VPL;     // (32 * VPL) / 4
+    constexpr int NCODE = 8 * VPL;
     constexpr int NW = VPL * W / 4;
     const int lane = threadIdx.x & 31;
-    const int R = (int)lds_u8(src);
+    const int R = (int)src.u8(0);
     if (R < TR::kFloor || R > TR::kFull) return false;
     const bool raw = R >= TR::kFull;
     const int s = raw ? 0 : ((8 - (R & 7)) & 7);
     const int req = (R + s) >> 3;
-    // (1) leading numbers: VPL/4 code bytes per lane
     uint32_t leads = 0;
 #pragma unroll
-    for (int q = 0; q < VPL / 4; q++) leads |= lds_u8(src + 1 + lane * (VPL / 4) + q) << (8 * q);
+    for (int q = 0; q < VPL / 4; q++) leads |= src.u8(1 + lane * (VPL / 4) + q) << (8 * q);
     uint32_t m = 0;
 #pragma unroll
     for (int i = 0; i < VPL; i++) {
@@ -288,18 +317,17 @@ __device__ inline bool decode_full(uint32_t src, uint32_t z, T mu, T (&out)[VPL]
     }
     const uint32_t incl = warp_incl_scan(m);
     if (1u + NCODE + __shfl_sync(0xffffffffu, incl, 31) != z) return false;
-    // (3) this lane's mid-bytes; value i takes the next m_i bytes of the run
     uint32_t run[NW];
-    run_load_s<NW>(src + 1 + NCODE + incl - m, run);
+    src.template run<NW>(1 + NCODE + incl - m, run);
     U own[VPL], cmk[VPL];
-    U M = ~U(0), D = 0;  // lane map: c -> (c & M) | D
+    U M = ~U(0), D = 0;
 #pragma unroll
     for (int i = 0; i < VPL; i++) {
         const int L = (leads >> (2 * i)) & 3;
         const int mi = req > L ? req - L : 0;
         U bytes;
         if (W == 4) {
-            bytes = run[0] & ~__funnelshift_lc(0u, 0xFFFFFFFFu, 8 * mi);  // low mi bytes (mi = 4: all)
+            bytes = run[0] & ~__funnelshift_lc(0u, 0xFFFFFFFFu, 8 * mi);
             run_drop4<NW>(run, mi);
         } else {
             bytes = ((U)run[0] | ((U)run[1] << 16 << 16)) & (mi >= 8 ? ~U(0) : ((U(1) << (8 * mi)) - U(1)));
@@ -307,12 +335,11 @@ __device__ inline bool decode_full(uint32_t src, uint32_t z, T mu, T (&out)[VPL]
             run_drop4<NW>(run, mi > 4 ? mi - 4 : 0);
         }
         own[i] = bytes << (8 * (W - req));
-        const int copy = L < req ? L : req;  // (2) bytes copied from the previous value
-        cmk[i] = ~(~U(0) >> (8 * copy));     // top `copy` bytes (copy <= 3 < W)
+        const int copy = L < req ? L : req;
+        cmk[i] = ~(~U(0) >> (8 * copy));
         M &= cmk[i];
         D = (D & cmk[i]) | own[i];
     }
-    // exclusive warp scan of lane maps -> the word carried into this lane (u_{-1} = 0)
     U cM = M, cD = D;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
@@ -322,7 +349,6 @@ __device__ inline bool decode_full(uint32_t src, uint32_t z, T mu, T (&out)[VPL]
     }
     U prev = __shfl_up_sync(0xffffffffu, cD, 1);
     if (lane == 0) prev = 0;
-    // (4) combine and overwrite the previous value, (5) left shift, add mu
 #pragma unroll
     for (int i = 0; i < VPL; i++) {
         const U w = (prev & cmk[i]) | own[i];
@@ -333,193 +359,224 @@ __device__ inline bool decode_full(uint32_t src, uint32_t z, T mu, T (&out)[VPL]
     return true;
 }
 
+#ifndef SZX_DMINB
+#define SZX_DMINB 3
+#endif
+#ifndef SZX_EXP
+#define SZX_EXP 0
+#endif
+#ifndef SZX_STCS
+#define SZX_STCS 0
+#endif
+#ifndef SZX_ROT
+#define SZX_ROT 0
+#endif
+// 16-byte store of decompressed output
+__device__ inline void st_out16(uint4* p, uint4 v) {
+#if SZX_STCS
+    __stcs(p, v);
+#else
+    *p = v;
+#endif
+}
+
 template <typename T, int VPL>
-__global__ void __launch_bounds__(DecodeCfg<T, VPL>::NT, DecodeCfg<T, VPL>::MINB)
-    k_decode(DPlan p, const uint8_t* __restrict__ in, T* __restrict__ y) {
+struct DecWCfg {
+#ifndef SZX_DSLOT
+#define SZX_DSLOT 3072
+#endif
+    static constexpr int NT = 256, NWARP = NT / 32;
+    static constexpr int SLOT = SZX_DSLOT;          // tile payload bytes staged in shared memory
+    static constexpr int SLOT_ALLOC = SLOT + 64;    // + over-read pad of the last block's run loads
+    static constexpr int SMEM = NWARP * 2 * SLOT_ALLOC;
+};
+
+// Per-tile metadata a warp needs before it can store anything.
+template <typename U>
+struct TileMeta {
+    uint32_t word;      // nonconstant bitmap of the tile's 32 blocks
+    uint32_t zl;        // lane r: zsize of the tile's r-th nonconstant block
+    uint64_t ncb;       // nonconstant index of the tile's first block
+    uint64_t base, end; // payload byte range
+    U mul;              // lane j: mu of block j
+};
+
+template <typename T, int VPL>
+__global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint8_t* __restrict__ in, T* __restrict__ y) {
     using TR = Traits<T>;
     using U = typename TR::U;
-    using C = DecodeCfg<T, VPL>;
-    extern __shared__ __align__(128) uint8_t smem[];
-    __shared__ __align__(8) uint64_t full_bar[C::STAGES], empty_bar[C::STAGES];
-    __shared__ __align__(16) uint16_t s_zw[C::STAGES][C::TB + 16];  // zsize window (TMA)
-    __shared__ uint32_t s_word[C::STAGES], s_sb[C::STAGES], s_zo[C::STAGES], s_ok[C::STAGES];
-    __shared__ uint64_t s_T[C::STAGES];
-
+    using C = DecWCfg<T, VPL>;
+    constexpr int W = TR::W;
+    constexpr int B = 32 * VPL;
+    constexpr int TB = kTileBlocks;
+    constexpr int MAXZ = 1 + B / 4 + W * B;
+    constexpr int NV = VPL * W / 16;  // 16-byte stores per lane per block
+    constexpr int QB = B * W / 16;    // 16-byte chunks per block
+    extern __shared__ __align__(16) uint8_t dsm[];
     pdl_wait();
     pdl_trigger();
-    const DHdr hd = read_dheader<TR::W>(in, p);
+    const DHdr hd = read_dheader<W>(in, p);
     if (!hd.ok) return;  // k_index has flagged it
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    if (threadIdx.x == 0) {
-        for (int s = 0; s < C::STAGES; s++) {
-            mbar_init(&full_bar[s], 1);
-            mbar_init(&empty_bar[s], C::NWARP);
-        }
-        fence_mbar_init();
-    }
-    __syncthreads();
-    const uint64_t G = gridDim.x;
+    const int lane = threadIdx.x & 31;
+    const uint32_t* bm = reinterpret_cast<const uint32_t*>(in + kHeaderBytes);
+    const uint16_t* zs = reinterpret_cast<const uint16_t*>(in + hd.off_zs);
+    const U* mus = reinterpret_cast<const U*>(in + p.off_mu);
+    const uint8_t* pl = in + hd.off_pl;
+    const uintptr_t lim = reinterpret_cast<uintptr_t>(in) + p.in_bytes;
+    const uint64_t nW_full = p.n / ((uint64_t)TB * B);
+    const uint32_t slot0 = smem_u32(dsm + (threadIdx.x >> 5) * 2 * C::SLOT_ALLOC);
 
-    if (warp == C::NWARP) {
-        // ---------------- producer: per tile, TMA bulk copies of the payload, the 32 mu
-        // values and the tile's zsize window; metadata fetched 32 tiles per round trip
-        const uintptr_t pl = reinterpret_cast<uintptr_t>(in + hd.off_pl);
-        const uintptr_t zsb = reinterpret_cast<uintptr_t>(in + hd.off_zs);
-        const uintptr_t lim = reinterpret_cast<uintptr_t>(in) + p.in_bytes;
-        const uintptr_t lim16 = lim & ~uintptr_t(15);
-        const uint32_t* bm = reinterpret_cast<const uint32_t*>(in + kHeaderBytes);
-        int i = 0;
-        for (uint64_t tb = blockIdx.x; tb < p.nW; tb += 32 * G) {
-            // lane l holds the metadata of tile tb + l*G
-            const uint64_t tl = tb + (uint64_t)lane * G;
-            uint32_t m_word = 0, m_ncb = 0;
-            uint64_t m_base = 0, m_end = 0;
-            if (tl < p.nW) {
-                m_word = bm[tl];
-                m_ncb = p.ncpre[tl];
-                m_base = p.tbase[tl];
-                m_end = p.tbase[tl + 1];
-            }
-            for (int j = 0; j < 32; j++, i++) {
-                const uint64_t t = tb + (uint64_t)j * G;
-                if (t >= p.nW) break;
-                uint32_t word = __shfl_sync(0xffffffffu, m_word, j);
-                const uint32_t ncb = __shfl_sync(0xffffffffu, m_ncb, j);
-                const uint64_t base = __shfl_sync(0xffffffffu, m_base, j);
-                const uint64_t end = __shfl_sync(0xffffffffu, m_end, j);
-                if (t == p.nW - 1 && (p.nB & 31)) word &= (1u << (p.nB & 31)) - 1u;
-                const uint32_t cnt = __popc(word);
-                const int s = i % C::STAGES;
-                mbar_wait(&empty_bar[s], ((i / C::STAGES) & 1) ^ 1);
-                uint8_t* pay = smem + (size_t)s * C::STAGE;
-                uint8_t* mub = pay + C::PAY;
-                const uint64_t Tb = end - base;
-                const bool ok = end >= base && Tb <= (uint64_t)C::TB * C::MAXZ && end <= hd.payload_bytes &&
-                                (uint64_t)ncb + cnt <= hd.nnc;
-                const uintptr_t a0 = pl + base;
-                const uintptr_t A = a0 & ~uintptr_t(15);
-                const uintptr_t E = ok ? ((a0 + Tb + 15) & ~uintptr_t(15)) : A;
-                const uintptr_t Eb = E < lim16 ? E : (lim16 > A ? lim16 : A);  // bulk part inside the buffer
-                const uint32_t bulk = (uint32_t)(Eb - A);
-                const uint64_t k0 = t * C::TB;
-                const bool mu_tma = (k0 + C::TB) <= p.nB;   // full tile of mu values
-                const uintptr_t za = (zsb + 2 * (uint64_t)ncb) & ~uintptr_t(15);
-                const uint32_t zbytes =
-                    (ok && cnt) ? (uint32_t)(((zsb + 2 * ((uint64_t)ncb + cnt) + 15) & ~uintptr_t(15)) - za) : 0u;
-                if (lane == 0) {
-                    mbar_expect_tx(&full_bar[s], bulk + (mu_tma ? (uint32_t)C::MUB : 0u) + zbytes);
-                    if (bulk) tma_load_1d(pay, reinterpret_cast<const void*>(A), bulk, &full_bar[s]);
-                    if (mu_tma) tma_load_1d(mub, in + p.off_mu + k0 * C::W, C::MUB, &full_bar[s]);
-                    if (zbytes) tma_load_1d(&s_zw[s][0], reinterpret_cast<const void*>(za), zbytes, &full_bar[s]);
-                    s_word[s] = word;
-                    s_sb[s] = (uint32_t)(a0 & 15);
-                    s_zo[s] = (uint32_t)((zsb + 2 * (uint64_t)ncb - za) >> 1);
-                    s_ok[s] = ok;
-                    s_T[s] = Tb;
-                }
-                // bytes of the last 16-byte chunk beyond the buffer's 16-byte floor
-                for (uintptr_t a = Eb + lane; a < E; a += 32)
-                    pay[a - A] = a < lim ? *reinterpret_cast<const uint8_t*>(a) : 0;
-                if (!mu_tma) {  // last, partial tile
-                    const U* mus = reinterpret_cast<const U*>(in + p.off_mu);
-                    if (k0 + lane < p.nB) reinterpret_cast<U*>(mub)[lane] = mus[k0 + lane];
-                }
-                __syncwarp();
-                if (lane == 0) mbar_arrive(&full_bar[s]);
-            }
+    auto load_meta = [&](uint64_t t, TileMeta<U>& m) {
+        uint32_t word = bm[t];
+        if (t == p.nW - 1 && (p.nB & 31)) word &= (1u << (p.nB & 31)) - 1u;
+        m.word = word;
+        m.ncb = p.ncpre[t];
+        m.base = p.tbase[t];
+        m.end = p.tbase[t + 1];
+        const uint64_t k0 = t * TB;
+        m.mul = k0 + lane < p.nB ? mus[k0 + lane] : U(0);
+    };
+    auto load_zl = [&](TileMeta<U>& m) {
+        const uint32_t cnt = __popc(m.word);
+        m.zl = ((uint32_t)lane < cnt && m.ncb + cnt <= hd.nnc) ? zs[m.ncb + lane] : 0u;
+    };
+    // Issue the cp.async copy of (the first SLOT bytes of) a tile's payload
+    // into slot `sl`; returns how many payload bytes, counted from the tile's
+    // first payload byte, the slot holds.
+    auto stage = [&](const TileMeta<U>& m, int sl) -> uint32_t {
+        if (!(m.end > m.base && m.end <= hd.payload_bytes) || (SZX_EXP & 8)) return 0;
+        const uintptr_t g0 = reinterpret_cast<uintptr_t>(pl + m.base);
+        const uintptr_t gA = g0 & ~uintptr_t(15);
+        uintptr_t gE = (reinterpret_cast<uintptr_t>(pl + m.end) + 15) & ~uintptr_t(15);
+        if (gE > gA + C::SLOT) gE = gA + C::SLOT;
+        const uint32_t sa = slot0 + sl * C::SLOT_ALLOC;
+        for (uintptr_t a = gA + 16 * lane; a < gE; a += 16 * 32) {
+            const uintptr_t rem = lim - a;
+            cp_async16_zfill(sa + (uint32_t)(a - gA), reinterpret_cast<const void*>(a), rem < 16 ? (uint32_t)rem : 16u);
         }
-        return;
-    }
+        return (uint32_t)(gE - g0);
+    };
+    // dynamic tile assignment: nonconstant-heavy tiles cost far more than
+    // constant ones, so static striding leaves warps idle at the end
+    auto grab = [&]() -> uint64_t {
+        uint32_t v = 0;
+        if (lane == 0) v = atomicAdd(&p.ctr[1], 1u);
+        return __shfl_sync(0xffffffffu, v, 0);
+    };
 
-    // ---------------- consumers
-    const uint32_t sbase = smem_u32(smem);
-    const uint64_t nW_full = p.n / ((uint64_t)C::TB * C::B);   // tiles whose 32 blocks are all full
-    constexpr int NV = VPL * C::W / 16;                          // 16-byte stores per lane per block
-    constexpr int QB = C::B * C::W / 16;                         // 16-byte chunks per block
-    const uint32_t below = (1u << lane) - 1u;
-    int i = 0;
-    for (uint64_t t = blockIdx.x; t < p.nW; t += G, i++) {
-        const int s = i % C::STAGES;
-        mbar_wait(&full_bar[s], (i / C::STAGES) & 1);
-        const uint32_t pay = sbase + s * C::STAGE;
-        const uint32_t mub = pay + C::PAY;
-        const uint32_t word = s_word[s];
+    uint64_t t = grab();
+    if (t >= p.nW) return;
+    TileMeta<U> cur, nx;
+    load_meta(t, cur);
+    load_zl(cur);
+    uint32_t cur_staged = stage(cur, 0);
+    cp_async_commit();
+    int sl = 0;
+    while (t < p.nW) {
+        const uint64_t tn = grab();
+        if (tn < p.nW) load_meta(tn, nx);
+        // validate the current tile's metadata
+        const uint32_t word = cur.word;
         const uint32_t cnt = __popc(word);
-        // zsize of the tile's nonconstant blocks (lane r holds the r-th); validate once
-        const uint32_t zl = (s_ok[s] && (uint32_t)lane < cnt) ? s_zw[s][s_zo[s] + lane] : 0u;
-        const bool zok = (uint32_t)lane >= cnt || (zl >= 2 && zl <= (uint32_t)C::MAXZ);
-        const bool ok = s_ok[s] && __all_sync(0xffffffffu, zok) && __reduce_add_sync(0xffffffffu, zl) == s_T[s];
-        const uint32_t mine = (word >> (warp * C::BPW)) & ((1u << C::BPW) - 1u);  // my nonconstant blocks
-        if (!ok) {
-            if (threadIdx.x == 0) set_corrupt(p.err);
-        } else if (t < nW_full) {
-            // full tile: every block holds B values
-            const uint32_t spay = pay + s_sb[s];
-            const uint32_t smu = mub + warp * C::BPW * C::W;
-            uint4* yq = reinterpret_cast<uint4*>(y + (t * C::TB + warp * C::BPW) * C::B + lane * VPL);
-            // constant blocks: retrieve with mu (Fig. 10, state 0)
-#pragma unroll
-            for (int j = 0; j < C::BPW; j++) {
-                if (!((mine >> j) & 1u)) {
-                    U mb = lds_u32(smu + j * C::W);
-                    if (C::W == 8) mb |= (U)lds_u32(smu + j * C::W + 4) << 16 << 16;
-                    T v[VPL];
-#pragma unroll
-                    for (int q = 0; q < VPL; q++) v[q] = TR::from(mb);
-#pragma unroll
-                    for (int q = 0; q < NV; q++) yq[j * QB + q] = reinterpret_cast<const uint4*>(v)[q];
-                }
-            }
-            // nonconstant blocks
-#pragma unroll 1
-            for (uint32_t m = mine; m; m &= m - 1) {
+        bool ok = cur.end >= cur.base && cur.end <= hd.payload_bytes && cur.ncb + cnt <= hd.nnc;
+        const uint32_t zl = cur.zl;
+        const bool zok = (uint32_t)lane >= cnt || (zl >= 2 && zl <= (uint32_t)MAXZ);
+        const uint32_t zincl = warp_incl_scan(zl);
+        ok = ok && __all_sync(0xffffffffu, zok) && __shfl_sync(0xffffffffu, zincl, 31) == cur.end - cur.base;
+        const uint32_t zoff = zincl - zl;
+        const uint64_t k0 = t * TB;
+        const bool full = t < nW_full;
+        // constant blocks of a full tile: retrieve with mu (Fig. 10, state 0)
+        if (ok && full && !(SZX_EXP & 1)) {
+            uint4* yq = reinterpret_cast<uint4*>(y + k0 * B + lane * VPL);
+#pragma unroll 2
+#if SZX_ROT
+            // start each tile at a different block so that concurrently active
+            // warps spread their stores over the address space
+            const uint32_t rot = (uint32_t)(t * 13) & 31u;
+            const uint32_t cw = (SZX_EXP & 4) ? ~0u : ~word;
+            for (uint32_t m = __funnelshift_r(cw, cw, rot); m; m &= m - 1) {
+                const int j = (__ffs(m) - 1 + rot) & 31;
+#else
+            for (uint32_t m = (SZX_EXP & 4) ? ~0u : ~word; m; m &= m - 1) {
                 const int j = __ffs(m) - 1;
-                const int idx = warp * C::BPW + j;
-                const uint32_t rank = __popc(word & ((1u << idx) - 1u));
-                const uint32_t off = __reduce_add_sync(0xffffffffu, (uint32_t)lane < rank ? zl : 0u);
-                const uint32_t z = __shfl_sync(0xffffffffu, zl, rank);
-                U mb = lds_u32(smu + j * C::W);
-                if (C::W == 8) mb |= (U)lds_u32(smu + j * C::W + 4) << 16 << 16;
+#endif
+                const U mb = __shfl_sync(0xffffffffu, cur.mul, j);
                 T v[VPL];
-                if (!decode_full<T, VPL>(spay + off, z, TR::from(mb), v)) {
-                    if (lane == 0) set_corrupt(p.err);
-                    continue;
-                }
 #pragma unroll
-                for (int q = 0; q < NV; q++) yq[j * QB + q] = reinterpret_cast<const uint4*>(v)[q];
+                for (int q = 0; q < VPL; q++) v[q] = TR::from(mb);
+#pragma unroll
+                for (int q = 0; q < NV; q++) st_out16(yq + j * QB + q, reinterpret_cast<const uint4*>(v)[q]);
             }
+        }
+        // prefetch the next tile's payload into the other slot
+        uint32_t nx_staged = 0;
+        if (tn < p.nW) {
+            load_zl(nx);
+            nx_staged = stage(nx, sl ^ 1);
+        }
+        cp_async_commit();
+        cp_async_wait<1>();
+        __syncwarp();
+        if (!ok) {
+            if (lane == 0) set_corrupt(p.err);
         } else {
-            // last (partial) tile: generic path with bounds and tail handling
-            const uint8_t* gpay = smem + (size_t)s * C::STAGE;
-            const U* gmu = reinterpret_cast<const U*>(gpay + C::PAY);
-            const int sb = (int)s_sb[s];
+            // nonconstant payloads: from the staging slot when the block lies
+            // inside the staged prefix, else straight from global memory
+            const uint32_t sbase = slot0 + sl * C::SLOT_ALLOC +
+                                   (uint32_t)(reinterpret_cast<uintptr_t>(pl + cur.base) & 15);
+            const uint8_t* gbase = pl + cur.base;
+            if (full) {
+                uint4* yq = reinterpret_cast<uint4*>(y + k0 * B + lane * VPL);
 #pragma unroll 1
-            for (int j = 0; j < C::BPW; j++) {
-                const int idx = warp * C::BPW + j;
-                const uint64_t k = t * C::TB + idx;
-                if (k >= p.nB) break;
-                const int len = (int)umin64(C::B, p.n - k * C::B);
-                const T mu = TR::from(gmu[idx]);
-                T v[VPL];
-                if (!((word >> idx) & 1u)) {
-#pragma unroll
-                    for (int q = 0; q < VPL; q++) v[q] = mu;
-                } else {
-                    const uint32_t rank = __popc(word & ((1u << idx) - 1u));
-                    const uint32_t off = __reduce_add_sync(0xffffffffu, (uint32_t)lane < rank ? zl : 0u);
-                    const uint32_t z = __shfl_sync(0xffffffffu, zl, rank);
-                    if (!decode_block<T, VPL>(gpay + sb + off, z, len, mu, v)) {
+                for (uint32_t m = (SZX_EXP & 2) ? 0u : word; m; m &= m - 1) {
+                    const int j = __ffs(m) - 1;
+                    const uint32_t r = __popc(word & ((1u << j) - 1u));
+                    const uint32_t off = __shfl_sync(0xffffffffu, zoff, r);
+                    const uint32_t z = __shfl_sync(0xffffffffu, zl, r);
+                    const T mu = TR::from(__shfl_sync(0xffffffffu, cur.mul, j));
+                    T v[VPL];
+                    bool good;
+                    if (off + z <= cur_staged) good = decode_full_g<T, VPL>(SrcS{sbase + off}, z, mu, v);
+                    else good = decode_full_g<T, VPL>(SrcG{gbase + off, lim}, z, mu, v);
+                    if (!good) {
                         if (lane == 0) set_corrupt(p.err);
                         continue;
                     }
+#pragma unroll
+                    for (int q = 0; q < NV; q++) st_out16(yq + j * QB + q, reinterpret_cast<const uint4*>(v)[q]);
                 }
-                store_lane<T, VPL>(y, p.n, k, lane, v);
+            } else {
+                // last (partial) tile: generic decoder, straight from global memory
+                for (int j = 0; j < TB; j++) {
+                    const uint64_t k = k0 + j;
+                    if (k >= p.nB) break;
+                    const int len = (int)umin64(B, p.n - k * B);
+                    const T mu = TR::from(__shfl_sync(0xffffffffu, cur.mul, j));
+                    T v[VPL];
+                    if (!((word >> j) & 1u)) {
+#pragma unroll
+                        for (int q = 0; q < VPL; q++) v[q] = mu;
+                    } else {
+                        const uint32_t r = __popc(word & ((1u << j) - 1u));
+                        const uint32_t off = __shfl_sync(0xffffffffu, zoff, r);
+                        const uint32_t z = __shfl_sync(0xffffffffu, zl, r);
+                        if (!decode_block_g<T, VPL>(SrcG{gbase + off, lim}, z, len, mu, v)) {
+                            if (lane == 0) set_corrupt(p.err);
+                            continue;
+                        }
+                    }
+                    store_lane<T, VPL>(y, p.n, k, lane, v);
+                }
             }
         }
-        (void)below;
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&empty_bar[s]);
+        __syncwarp();  // slot `sl` is refilled two tiles from now
+        cur = nx;
+        cur_staged = nx_staged;
+        sl ^= 1;
+        t = tn;
     }
+    cp_async_wait<0>();
 }
 
 }  // namespace szx

@@ -138,13 +138,23 @@ __device__ inline uint64_t warp_sum64(uint64_t v) {
     return v;
 }
 // inclusive prefix sum over the warp
+// (shfl.up's own in-range predicate guards the add: one SHFL + one IADD per step)
+template <int O>
+__device__ inline uint32_t shfl_up_add(uint32_t v) {
+    asm volatile(
+        "{\n\t.reg .u32 t;\n\t.reg .pred p;\n\t"
+        "shfl.sync.up.b32 t|p, %0, %1, 0, -1;\n\t"
+        "@p add.u32 %0, %0, t;\n\t}"
+        : "+r"(v)
+        : "n"(O));
+    return v;
+}
 __device__ inline uint32_t warp_incl_scan(uint32_t v) {
-    const int lane = threadIdx.x & 31;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        uint32_t t = __shfl_up_sync(0xffffffffu, v, o);
-        if (lane >= o) v += t;
-    }
+    v = shfl_up_add<1>(v);
+    v = shfl_up_add<2>(v);
+    v = shfl_up_add<4>(v);
+    v = shfl_up_add<8>(v);
+    v = shfl_up_add<16>(v);
     return v;
 }
 
@@ -158,6 +168,10 @@ __device__ inline void pdl_trigger() { asm volatile("griddepcontrol.launch_depen
 // ---------------------------------------------------------------- cp.async
 __device__ inline void cp_async16(uint32_t saddr, const void* g) {
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(saddr), "l"(g) : "memory");
+}
+// 16-byte copy of which only the first `src_bytes` (1..16) are read; the rest is zero-filled
+__device__ inline void cp_async16_zfill(uint32_t saddr, const void* g, uint32_t src_bytes) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(saddr), "l"(g), "r"(src_bytes) : "memory");
 }
 __device__ inline void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 template <int N>

@@ -15,7 +15,7 @@ from dataclasses import dataclass
 import torch
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libszx_b200.so")
+LIB_PATH = os.environ.get("SZX_LIB", os.path.join(_PKG, "libszx_b200.so"))  # SZX_LIB: experiment builds
 
 F32, F64 = 0, 1
 ABS, REL = 0, 1
