@@ -180,10 +180,27 @@ int check_compress_args(const void* d_in, szx_dtype_t dt, uint64_t n, szx_ebmode
     return SZX_OK;
 }
 
+#ifndef SZX_CARVE
+#define SZX_CARVE 0
+#endif
+// every kernel asks for the same L1/shared split, so consecutive kernels do
+// not make the SMs drain and reconfigure the carve-out
+template <typename K>
+void carve(K k) {
+    if (SZX_CARVE) cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, SZX_CARVE);
+}
+
 template <typename T, int VPL>
 void set_smem_attrs() {
     static bool done = false;
     if (done) return;
+    constexpr int UNR = 128 / (VPL * (int)sizeof(T)) > 0 ? 128 / (VPL * (int)sizeof(T)) : 1;
+    carve(k_block_stats<T, VPL, UNR>);
+    carve(k_classify<T>);
+    carve(k_enc_size<T, VPL>);
+    carve(k_zscan<Traits<T>::W>);
+    carve(k_enc_write<T, VPL>);
+    carve(k_decode_w<T, VPL>);
     cudaFuncSetAttribute(k_enc_write<T, VPL>, cudaFuncAttributeMaxDynamicSharedMemorySize, WriteCfg<T, VPL>::SMEM);
     cudaFuncSetAttribute(k_enc_size<T, VPL>, cudaFuncAttributeMaxDynamicSharedMemorySize, SizeCfg<T, VPL>::SMEM);
 
@@ -194,6 +211,7 @@ void set_smem_attrs() {
 // UNR blocks (128 bytes per lane) of loads in flight
 template <typename T, int VPL>
 void enqueue_stats(const void* d_in, const Plan& p, int want_range, cudaStream_t s) {
+    set_smem_attrs<T, VPL>();
     constexpr int UNR = 128 / (VPL * (int)sizeof(T)) > 0 ? 128 / (VPL * (int)sizeof(T)) : 1;
     static int occ = 0;
     if (!occ) {
@@ -295,16 +313,17 @@ int64_t finish_sync(cudaStream_t s, const uint64_t* d_val, uint64_t* out_val) {
 // ------------------------------------------------------------ decompress layout
 // Sized from the shape only (n, b): the number of nonconstant blocks is read
 // from the stream header on the device, so the layout covers nNC <= nB.
+constexpr uint64_t kMaxDecodeGrid = 2048;  // co-resident CTAs of k_decode_w (slot arrays)
+
 struct DLayout {
-    uint64_t nB, nW, nTI;
+    uint64_t nB, nW;
     uint64_t zero_bytes, off_ncpre, off_tbase, total;
 };
 DLayout dlayout(uint64_t n, uint32_t b) {
     DLayout L{};
     L.nB = cdiv(n, b);
     L.nW = cdiv(L.nB, 32);
-    L.nTI = cdiv(L.nW, kIndexTiles);
-    L.zero_bytes = al16(16 + 16 + 16 * L.nTI);  // ctr[2], err, status_a, status_z
+    L.zero_bytes = 16 + 16 + 4 * 8 * kMaxDecodeGrid;  // ctr[4], err, slot_a, res_a, slot_z, res_z
     L.off_ncpre = L.zero_bytes;
     L.off_tbase = al16(L.off_ncpre + 4 * L.nW + 4);
     L.total = al16(L.off_tbase + 8 * (L.nW + 1)) + 256;
@@ -357,8 +376,10 @@ int enqueue_decompress(const void* d_in, uint64_t in_bytes, const szx_header_t* 
     p.dtype = h->dtype;
     p.ctr = reinterpret_cast<uint32_t*>(ws);
     p.err = reinterpret_cast<int32_t*>(ws + 16);
-    p.status_a = reinterpret_cast<uint64_t*>(ws + 32);
-    p.status_z = p.status_a + L.nTI;
+    p.slot_a = reinterpret_cast<uint64_t*>(ws + 32);
+    p.res_a = p.slot_a + kMaxDecodeGrid;
+    p.slot_z = p.res_a + kMaxDecodeGrid;
+    p.res_z = p.slot_z + kMaxDecodeGrid;
     p.ncpre = reinterpret_cast<uint32_t*>(ws + L.off_ncpre);
     p.tbase = reinterpret_cast<uint64_t*>(ws + L.off_tbase);
     *d_err_out = p.err;
@@ -368,8 +389,9 @@ int enqueue_decompress(const void* d_in, uint64_t in_bytes, const szx_header_t* 
     dispatch((szx_dtype_t)h->dtype, h->block_size, [&](auto tag, auto vpl) {
         using T = decltype(tag);
         constexpr int V = decltype(vpl)::value;
-        launch("k_index", s, [&] { k_index<Traits<T>::W><<<(unsigned)L.nTI, 256, 0, s>>>(p, in); });
-        // one warp per 32-block tile, grid-stride; enough CTAs for full occupancy
+        set_smem_attrs<T, V>();
+        // persistent, co-resident grid (index phase, grid barrier, then one
+        // warp per 32-block tile)
         static int occ = 0;
         if (!occ) {
             cudaFuncSetAttribute(k_decode_w<T, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, DecWCfg<T, V>::SMEM);
@@ -379,6 +401,7 @@ int enqueue_decompress(const void* d_in, uint64_t in_bytes, const szx_header_t* 
         uint64_t grid = cdiv(L.nW, 8);
         const uint64_t cap = (uint64_t)sm_count() * occ;
         if (grid > cap) grid = cap;
+        if (grid > kMaxDecodeGrid) grid = kMaxDecodeGrid;
         launch("k_decode", s, [&] {
             launch_pdl(k_decode_w<T, V>, dim3((unsigned)grid), dim3(256), DecWCfg<T, V>::SMEM, s, p, in, static_cast<T*>(d_out));
         });

@@ -414,6 +414,50 @@ __device__ inline void encode_block(const T (&xv)[VPL], int cnt, int len, T mu, 
     lc.z = 1 + (uint32_t)((len + 3) / 4) + __shfl_sync(0xffffffffu, incl, 31);
 }
 
+// Size of one FULL nonconstant block (the size pass needs z_k and the final
+// R only): same R / guard / escalation as encode_block, but the mid-byte
+// count is a warp sum (one REDUX) instead of a scan and no codes are kept.
+template <typename T, int VPL>
+__device__ inline uint32_t size_block(const T (&xv)[VPL], T mu, int& R, bool proven, double eb) {
+    using TR = Traits<T>;
+    using U = typename TR::U;
+    constexpr int W = TR::W;
+    const int lane = threadIdx.x & 31;
+    int s, req;
+    bool raw;
+    bool check = !proven;
+    U u[VPL];
+    for (;;) {
+        raw = R >= TR::kFull;
+        if (raw) { R = TR::kFull; mu = T(0); }
+        s = raw ? 0 : ((8 - (R & 7)) & 7);
+        req = (R + s) >> 3;
+#pragma unroll
+        for (int i = 0; i < VPL; i++) u[i] = (raw ? TR::bits(xv[i]) : TR::bits(TR::sub(xv[i], mu))) >> s;
+        if (raw || !check) break;
+        const U keep = ~((U(1) << (8 * W - R)) - U(1));
+        bool ok = true;
+#pragma unroll
+        for (int i = 0; i < VPL; i++) {
+            const T xp = TR::add(TR::from((u[i] << s) & keep), mu);
+            ok &= fabs(__dsub_rn((double)xv[i], (double)xp)) <= eb;
+        }
+        if (__all_sync(0xffffffffu, ok)) break;
+        R += 1;
+    }
+    U prev = __shfl_up_sync(0xffffffffu, u[VPL - 1], 1);
+    if (lane == 0) prev = 0;
+    uint32_t m = 0;
+#pragma unroll
+    for (int i = 0; i < VPL; i++) {
+        int L = TR::clz(u[i] ^ prev) >> 3;
+        L = L > 3 ? 3 : L;
+        m += req > L ? req - L : 0;
+        prev = u[i];
+    }
+    return 1 + (uint32_t)(8 * VPL) + warp_sum(m);
+}
+
 // Write the block payload [R][codes][mid-bytes] into shared memory at dst.
 template <typename T, int VPL>
 __device__ inline void pack_block(const typename Traits<T>::U (&u)[VPL], const LaneCode& lc, int cnt, int len,
@@ -574,31 +618,64 @@ __global__ void __launch_bounds__(256) k_enc_size(const T* __restrict__ x, Plan 
             }
             __syncwarp();
             const uint32_t st = sbuf + (b & 1) * C::NB * C::BW;
+            // full blocks two at a time: independent instruction streams for ILP
 #pragma unroll 1
-            for (int j = 0; j < C::NB; j++) {
+            for (int j = 0; j < C::NB; j += 2) {
                 const int l = b * C::NB + j;
                 const uint64_t nc = g0 + l;
-                const uint32_t k = __shfl_sync(0xffffffffu, mk, l);
-                const T mu = TR::from(__shfl_sync(0xffffffffu, mmu, l));
-                const uint32_t rec = __shfl_sync(0xffffffffu, mrec, l);
                 if (nc >= c1) break;
-                T xv[VPL];
-                U uu[VPL];
-                LaneCode lc;
-                if (k < nBfull) {
+                const bool two = nc + 1 < c1;
+                const uint32_t k0 = __shfl_sync(0xffffffffu, mk, l);
+                const uint32_t k1 = __shfl_sync(0xffffffffu, mk, l + 1);
+                const T mu0 = TR::from(__shfl_sync(0xffffffffu, mmu, l));
+                const T mu1 = TR::from(__shfl_sync(0xffffffffu, mmu, l + 1));
+                const uint32_t rec0 = __shfl_sync(0xffffffffu, mrec, l);
+                const uint32_t rec1 = __shfl_sync(0xffffffffu, mrec, l + 1);
+                if (k0 < nBfull && (!two || k1 < nBfull)) {
+                    T x0[VPL], x1[VPL];
 #pragma unroll
-                    for (int q = 0; q < C::QV; q++)
-                        reinterpret_cast<uint4*>(xv)[q] = lds_u128(st + j * C::BW + (lane * C::QV + q) * 16);
-                    encode_block<T, VPL>(xv, VPL, B, mu, (int)(rec & 0x7F), (rec & 0x80) != 0, eb, uu, lc);
-                } else {  // the partial tail block
-                    const int cnt = load_lane<T, VPL>(x, p.n, k, lane, xv);
-                    const int len = (int)(p.n - (uint64_t)k * B);
-                    encode_block<T, VPL>(xv, cnt, len, mu, (int)(rec & 0x7F), (rec & 0x80) != 0, eb, uu, lc);
+                    for (int q = 0; q < C::QV; q++) {
+                        reinterpret_cast<uint4*>(x0)[q] = lds_u128(st + j * C::BW + (lane * C::QV + q) * 16);
+                        reinterpret_cast<uint4*>(x1)[q] = lds_u128(st + (j + 1) * C::BW + (lane * C::QV + q) * 16);
+                    }
+                    int R0 = (int)(rec0 & 0x7F), R1 = (int)(rec1 & 0x7F);
+                    const uint32_t z0 = size_block<T, VPL>(x0, mu0, R0, (rec0 & 0x80) != 0, eb);
+                    const uint32_t z1 = two ? size_block<T, VPL>(x1, mu1, R1, (rec1 & 0x80) != 0, eb) : 0u;
+                    if (lane == 0) {
+                        zsize[nc] = (uint16_t)z0;
+                        p.ncR[nc] = (uint8_t)R0;
+                        if (R0 >= TR::kFull) mus[k0] = 0;  // raw (NaN, Formula 4 or escalation): mu = +0 (R15)
+                        if (two) {
+                            zsize[nc + 1] = (uint16_t)z1;
+                            p.ncR[nc + 1] = (uint8_t)R1;
+                            if (R1 >= TR::kFull) mus[k1] = 0;
+                        }
+                    }
+                    continue;
                 }
-                if (lane == 0) {
-                    zsize[nc] = (uint16_t)lc.z;
-                    p.ncR[nc] = (uint8_t)lc.R;
-                    if (lc.R >= TR::kFull) mus[k] = 0;  // raw (NaN, Formula 4 or escalation): mu = +0 (R15)
+                // a pair holding the partial tail block: one block at a time
+                for (int h = 0; h < (two ? 2 : 1); h++) {
+                    const uint32_t k = h ? k1 : k0;
+                    const T mu = h ? mu1 : mu0;
+                    const uint32_t rec = h ? rec1 : rec0;
+                    T xv[VPL];
+                    U uu[VPL];
+                    LaneCode lc;
+                    if (k < nBfull) {
+#pragma unroll
+                        for (int q = 0; q < C::QV; q++)
+                            reinterpret_cast<uint4*>(xv)[q] = lds_u128(st + (j + h) * C::BW + (lane * C::QV + q) * 16);
+                        encode_block<T, VPL>(xv, VPL, B, mu, (int)(rec & 0x7F), (rec & 0x80) != 0, eb, uu, lc);
+                    } else {
+                        const int cnt = load_lane<T, VPL>(x, p.n, k, lane, xv);
+                        const int len = (int)(p.n - (uint64_t)k * B);
+                        encode_block<T, VPL>(xv, cnt, len, mu, (int)(rec & 0x7F), (rec & 0x80) != 0, eb, uu, lc);
+                    }
+                    if (lane == 0) {
+                        zsize[nc + h] = (uint16_t)lc.z;
+                        p.ncR[nc + h] = (uint8_t)lc.R;
+                        if (lc.R >= TR::kFull) mus[k] = 0;
+                    }
                 }
             }
             __syncwarp();

@@ -1,23 +1,24 @@
 // szx_decompress.cuh -- SZx decompression kernels for sm_100a.
 //
-//   k_index   (K5a) the paper's "prefix-sum step to compute the starting
-//             location of each block", as two chained
-//             single-pass decoupled look-back scans per CTA of 256 tiles
-//             (tile = 32 blocks = one bitmap word):
-//               (a) nonconstant index of each tile = prefix of popcounts,
-//               (b) payload byte offset of each tile = prefix of its zsize
-//                   sums (the CTA's zsize range is staged in shared memory).
-//             Totals are validated against the header (nNC, payload size).
-//   k_decode_w (K5) a warp per 32-block tile (grid-stride): metadata, mu
-//             values, zsize entries and the nonconstant payloads are read
-//             straight from global memory; the values are rebuilt with the
-//             five steps of Fig. 10 and written with 16-byte
-//             stores.  The leading-byte dependence chains
-//             (Challenge 2) are resolved with a warp scan of
-//             byte-mask transfer functions instead of the paper's log-step
-//             index propagation: a lane's values map an
-//             incoming previous word c to (c & M) | D, and composing such
-//             maps is associative.
+// One persistent kernel, k_decode_w, whose grid is co-resident (<= SMs x
+// occupancy):
+//   (K5a) index phase -- the paper's "prefix-sum step to compute the starting
+//         location of each block": per tile (32 blocks = one
+//         bitmap word) its nonconstant index (prefix of popcounts) and its
+//         payload byte offset (prefix of zsize sums).  Each CTA owns a
+//         contiguous tile range; two grid-wide prefixes over CTA aggregates
+//         replace chained look-backs.  Totals are validated against the
+//         header (nNC, payload size).  A grid barrier follows.
+//   (K5)  decode phase -- a warp per 32-block tile (dynamic assignment, two
+//         tiles in flight): metadata, mu values and zsize entries from
+//         global memory, the tile's payload staged in shared memory with
+//         cp.async; values rebuilt with the five steps of Fig. 10
+//          and written with 16-byte stores.  The leading-byte
+//         dependence chains (Challenge 2) are resolved with a
+//         warp scan of byte-mask transfer functions instead of the paper's
+//         log-step index propagation: a lane's values map an
+//         incoming previous word c to (c & M) | D, and composing such maps is
+//         associative.
 #pragma once
 
 #include "szx_device.cuh"
@@ -30,9 +31,11 @@ struct DPlan {
     uint64_t n, nB, nW, in_bytes;
     uint64_t off_mu;
     uint32_t b, dtype;
-    uint32_t* ctr;             // [2] init 0: k_index tile ticket, k_decode_w tile counter
-    uint64_t* status_a;        // init 0
-    uint64_t* status_z;        // init 0
+    uint32_t* ctr;             // [4] init 0: [0] [3] prefix arrivals, [1] tile counter, [2] grid barrier
+    uint64_t* slot_a;          // [grid] per-CTA nonconstant counts
+    uint64_t* res_a;           // [grid] init 0: their exclusive prefixes
+    uint64_t* slot_z;          // [grid] per-CTA payload byte counts
+    uint64_t* res_z;           // [grid] init 0: their exclusive prefixes
     uint32_t* ncpre;           // [nW]      nonconstant index of each tile's first block
     uint64_t* tbase;           // [nW + 1]  payload offset of each tile (tbase[nW] = total)
     int32_t* err;              // 0 ok, else SZX_ECORRUPT
@@ -86,60 +89,112 @@ __device__ inline uint64_t cta_scan256(uint64_t v, uint64_t* agg, uint64_t* s_w 
     return wpre + incl - v;
 }
 
-constexpr int kIndexTiles = 256;  // tiles (bitmap words) per k_index CTA
+// --------------------------------------------------------------- index phase
+// Decoder prologue (Fig. 10 needs, for every 32-block tile t, where its
+// nonconstant blocks start in the zsize array and in the payload):
+//   ncpre[t] = popcount of the bitmap words before t,
+//   tbase[t] = sum of the zsizes of the nonconstant blocks before t.
+// CTA c owns a contiguous range of tiles.  Two grid-wide prefixes over CTA
+// aggregates (grid_excl_prefix: the grid is co-resident) give the CTA its
+// starting nonconstant index and payload offset; it then scans its range in
+// chunks of 256 tiles.  Run by all 256 threads; s_zs: 256*32 u16 scratch.
+#ifndef SZX_DMINB
+#define SZX_DMINB 3
+#endif
+#ifndef SZX_EXP
+#define SZX_EXP 0
+#endif
+#ifndef SZX_STCS
+#define SZX_STCS 0
+#endif
+#ifndef SZX_ROT
+#define SZX_ROT 0
+#endif
+constexpr int kIndexChunk = 256;
 
-template <int W>
-__global__ void __launch_bounds__(256) k_index(DPlan p, const uint8_t* __restrict__ in) {
-    __shared__ uint64_t s_tile, s_ga, s_gb, s_w[8];
-    __shared__ uint16_t s_zs[kIndexTiles * 32];
-    const DHdr hd = read_dheader<W>(in, p);
-    if (!hd.ok) {
-        if (blockIdx.x == 0 && threadIdx.x == 0) set_corrupt(p.err);
-        return;
-    }
-    if (threadIdx.x == 0) s_tile = atomicAdd(&p.ctr[0], 1u);
-    __syncthreads();
-    const uint64_t t = s_tile;
-    const uint64_t ntiles = (p.nW + kIndexTiles - 1) / kIndexTiles;
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const uint64_t w = t * kIndexTiles + threadIdx.x;
-    // (a) nonconstant index of each tile
-    uint32_t word = w < p.nW ? reinterpret_cast<const uint32_t*>(in + kHeaderBytes)[w] : 0u;
-    if (w == p.nW - 1 && (p.nB & 31)) word &= (1u << (p.nB & 31)) - 1u;  // ignore padding bits
-    const uint32_t cnt = __popc(word);
-    uint64_t aggA;
-    const uint64_t exA = cta_scan256(cnt, &aggA, s_w);
-    if (warp == 0) {
-        const uint64_t e = lookback_exclusive(p.status_a, t, aggA);
-        if (lane == 0) s_ga = e;
-    }
-    __syncthreads();
-    const uint64_t GA = s_ga;
-    const uint64_t ncb = GA + exA;
-    if (w < p.nW) p.ncpre[w] = (uint32_t)ncb;
-    bool ok = GA + aggA <= hd.nnc;
-    // (b) stage this CTA's zsize entries [GA, GA + aggA) and sum per tile
-    const uint16_t* zs = reinterpret_cast<const uint16_t*>(in + hd.off_zs);
-    const uint64_t nz = ok ? aggA : 0;
-    for (uint64_t j = threadIdx.x; j < nz; j += 256) s_zs[j] = zs[GA + j];
-    __syncthreads();
-    uint64_t sum = 0;
-    if (ok)
-        for (uint32_t j = 0; j < cnt; j++) sum += s_zs[exA + j];
-    uint64_t aggB;
-    const uint64_t exB = cta_scan256(sum, &aggB, s_w);
-    if (warp == 0) {
-        const uint64_t e = lookback_exclusive(p.status_z, t, aggB);
-        if (lane == 0) {
-            s_gb = e;
-            if (t == ntiles - 1) {
-                p.tbase[p.nW] = e + aggB;
-                if (GA + aggA != hd.nnc || e + aggB != hd.payload_bytes) set_corrupt(p.err);
-            }
+// Copy zs[i0, i0 + cnt) (cnt <= 32 * kIndexChunk) into shared memory with
+// aligned 16-byte loads.  The zsize section is 16-byte aligned and padded to
+// a multiple of 16 bytes, so the rounded-out loads stay inside it.
+__device__ inline void stage_u16(uint16_t* s_dst, const uint16_t* __restrict__ zs, uint64_t i0, uint64_t cnt) {
+    const uint64_t a = i0 & ~uint64_t(7);
+    const uint32_t head = (uint32_t)(i0 - a);
+    const uint32_t nq = (uint32_t)((head + cnt + 7) / 8);
+    for (uint32_t q = threadIdx.x; q < nq; q += kIndexChunk) {
+        const uint4 v = *reinterpret_cast<const uint4*>(zs + a + 8 * q);
+        const uint32_t e[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+        for (int k = 0; k < 8; k++) {
+            const int64_t d = (int64_t)(8 * q + k) - head;
+            if (d >= 0 && (uint64_t)d < cnt) s_dst[d] = (uint16_t)(e[k >> 1] >> (16 * (k & 1)));
         }
     }
-    if (!__syncthreads_and(ok ? 1 : 0) && threadIdx.x == 0) set_corrupt(p.err);
-    if (w < p.nW) p.tbase[w] = s_gb + exB;
+}
+
+template <int W>
+__device__ inline void index_phase(const DPlan& p, const uint8_t* __restrict__ in, const DHdr& hd,
+                                   uint16_t* s_zs, uint64_t* s_w) {
+    const uint64_t G = gridDim.x, c = blockIdx.x;
+    const uint64_t w0 = p.nW * c / G, w1 = p.nW * (c + 1) / G;
+    const uint32_t* bm = reinterpret_cast<const uint32_t*>(in + kHeaderBytes);
+    const uint16_t* zs = reinterpret_cast<const uint16_t*>(in + hd.off_zs);
+    auto word_at = [&](uint64_t w) -> uint32_t {
+        uint32_t x = bm[w];
+        if (w == p.nW - 1 && (p.nB & 31)) x &= (1u << (p.nB & 31)) - 1u;  // ignore padding bits
+        return x;
+    };
+    // (1) nonconstant blocks in the range -> starting nonconstant index
+    uint64_t cnt = 0;
+    for (uint64_t w = w0 + threadIdx.x; w < w1; w += kIndexChunk) cnt += __popc(word_at(w));
+    const uint64_t aggA = cta_sum64(cnt, s_w);
+    if (SZX_EXP & 128) { if (threadIdx.x == 0 && aggA == 12345) p.ncpre[0] = 1; return; }
+    const uint64_t exA = grid_excl_prefix(p.slot_a, p.res_a, &p.ctr[0], aggA, s_w);
+    if (SZX_EXP & 64) { if (threadIdx.x == 0 && exA == 12345) p.ncpre[0] = 1; return; }
+    const bool ok = exA + aggA <= hd.nnc;
+    // (2) their payload bytes -> starting payload offset.  A range of at most
+    // one chunk keeps its zsizes in shared memory for step (3).
+    const bool one = w1 - w0 <= (uint64_t)kIndexChunk;
+    uint64_t zsum = 0;
+    if (ok) {
+        if (one) {
+            stage_u16(s_zs, zs, exA, aggA);
+            __syncthreads();
+            for (uint32_t j = threadIdx.x; j < aggA; j += kIndexChunk) zsum += s_zs[j];
+        } else {
+            for (uint64_t i = exA + threadIdx.x; i < exA + aggA; i += kIndexChunk) zsum += zs[i];
+        }
+    }
+    const uint64_t aggZ = cta_sum64(zsum, s_w);
+    const uint64_t exZ = grid_excl_prefix(p.slot_z, p.res_z, &p.ctr[3], aggZ, s_w);
+    // (3) per tile: ncpre and tbase
+    uint64_t runA = exA, runZ = exZ;
+    for (uint64_t wc = w0; wc < w1; wc += kIndexChunk) {
+        const uint64_t w = wc + threadIdx.x;
+        const uint32_t word = w < w1 ? word_at(w) : 0u;
+        const uint32_t cw = __popc(word);
+        uint64_t tot;
+        const uint64_t ex = cta_scan256(cw, &tot, s_w);
+        if (w < w1) p.ncpre[w] = (uint32_t)(runA + ex);
+        if (!one) {
+            if (ok) stage_u16(s_zs, zs, runA, tot);
+            __syncthreads();
+        }
+        uint64_t sum = 0;
+        if (ok)
+            for (uint32_t j = 0; j < cw; j++) sum += s_zs[ex + j];
+        uint64_t totz;
+        const uint64_t exz = cta_scan256(sum, &totz, s_w);
+        if (w < w1) p.tbase[w] = runZ + exz;
+        runA += tot;
+        runZ += totz;
+        __syncthreads();  // s_zs is refilled by the next chunk
+    }
+    if (threadIdx.x == 0) {
+        if (!ok) set_corrupt(p.err);
+        if (c == G - 1) {
+            p.tbase[p.nW] = runZ;
+            if (runA != hd.nnc || runZ != hd.payload_bytes) set_corrupt(p.err);
+        }
+    }
 }
 
 template <typename T, int VPL>
@@ -359,18 +414,6 @@ __device__ inline bool decode_full_g(const Src src, uint32_t z, T mu, T (&out)[V
     return true;
 }
 
-#ifndef SZX_DMINB
-#define SZX_DMINB 3
-#endif
-#ifndef SZX_EXP
-#define SZX_EXP 0
-#endif
-#ifndef SZX_STCS
-#define SZX_STCS 0
-#endif
-#ifndef SZX_ROT
-#define SZX_ROT 0
-#endif
 // 16-byte store of decompressed output
 __device__ inline void st_out16(uint4* p, uint4 v) {
 #if SZX_STCS
@@ -389,6 +432,7 @@ struct DecWCfg {
     static constexpr int SLOT = SZX_DSLOT;          // tile payload bytes staged in shared memory
     static constexpr int SLOT_ALLOC = SLOT + 64;    // + over-read pad of the last block's run loads
     static constexpr int SMEM = NWARP * 2 * SLOT_ALLOC;
+    static_assert(SMEM >= kIndexChunk * 32 * 2, "index-phase scratch aliases the slots");
 };
 
 // Per-tile metadata a warp needs before it can store anything.
@@ -413,10 +457,20 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
     constexpr int NV = VPL * W / 16;  // 16-byte stores per lane per block
     constexpr int QB = B * W / 16;    // 16-byte chunks per block
     extern __shared__ __align__(16) uint8_t dsm[];
+    __shared__ uint64_t s_w[32];
     pdl_wait();
     pdl_trigger();
     const DHdr hd = read_dheader<W>(in, p);
-    if (!hd.ok) return;  // k_index has flagged it
+    if (!hd.ok) {  // every CTA sees the same header: all leave
+        if (blockIdx.x == 0 && threadIdx.x == 0) set_corrupt(p.err);
+        return;
+    }
+    // index phase (the shared staging slots double as its scratch), then a
+    // grid barrier: tiles are decoded by whichever warp grabs them
+    index_phase<W>(p, in, hd, reinterpret_cast<uint16_t*>(dsm), s_w);
+    if (SZX_EXP & 32) return;
+    grid_barrier(&p.ctr[2]);
+    if (SZX_EXP & 16) return;
     const int lane = threadIdx.x & 31;
     const uint32_t* bm = reinterpret_cast<const uint32_t*>(in + kHeaderBytes);
     const uint16_t* zs = reinterpret_cast<const uint16_t*>(in + hd.off_zs);

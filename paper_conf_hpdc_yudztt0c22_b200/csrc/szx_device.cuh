@@ -430,4 +430,94 @@ __device__ inline uint64_t lookback_exclusive(uint64_t* status, uint64_t tile, u
     return excl;
 }
 
+// ------------------------------------------------- co-resident grid helpers
+// Used by persistent kernels whose grid never exceeds the number of CTAs the
+// device can hold at once (grid <= SMs x occupancy, set on the host), so every
+// CTA is running and spinning on another CTA's flag cannot deadlock.
+
+__device__ inline uint32_t ld_acquire_u32(const uint32_t* p) {
+    uint32_t v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
+// Sum over the CTA (any blockDim that is a multiple of 32, <= 1024); result
+// in every thread.  s_w: shared scratch of 32 u64.
+__device__ inline uint64_t cta_sum64(uint64_t v, uint64_t* s_w) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarp = blockDim.x >> 5;
+    v = warp_sum64(v);
+    __syncthreads();  // s_w may still be read by a previous call
+    if (lane == 0) s_w[warp] = v;
+    __syncthreads();
+    uint64_t t = 0;
+    for (int i = 0; i < nwarp; i++) t += s_w[i];
+    return t;
+}
+
+// Grid-wide exclusive prefix of one aggregate per CTA, in CTA order.  Each
+// CTA stores its aggregate and takes an arrival ticket; the last CTA to
+// arrive scans all aggregates and publishes each CTA's prefix (flag bit 63)
+// in res[]; every CTA waits on its own entry.  Cost: one atomic per CTA and
+// about three round trips, with no chained look-back and no all-to-all
+// polling.  `res` [gridDim.x] and `*arrive` must be zero.
+constexpr uint64_t kSlotFlag = 1ull << 63;
+__device__ inline uint64_t grid_excl_prefix(uint64_t* slots, uint64_t* res, uint32_t* arrive, uint64_t agg,
+                                            uint64_t* s_w /*[32]*/) {
+    __shared__ uint32_t s_last;
+    __shared__ uint64_t s_val;
+    const uint32_t G = gridDim.x;
+    if (threadIdx.x == 0) {
+        st_relaxed(&slots[blockIdx.x], agg);
+        __threadfence();
+        s_last = atomicAdd(arrive, 1u) == G - 1;
+    }
+    __syncthreads();
+    if (s_last) {
+        __threadfence();
+        uint64_t run = 0;
+        for (uint32_t b0 = 0; b0 < G; b0 += blockDim.x) {
+            const uint32_t i = b0 + threadIdx.x;
+            const uint64_t v = i < G ? ld_relaxed(&slots[i]) : 0;
+            // CTA exclusive scan of v
+            const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarp = blockDim.x >> 5;
+            uint64_t incl = v;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint64_t t = __shfl_up_sync(0xffffffffu, incl, o);
+                if (lane >= o) incl += t;
+            }
+            __syncthreads();
+            if (lane == 31) s_w[warp] = incl;
+            __syncthreads();
+            uint64_t wpre = 0, tot = 0;
+            for (int k = 0; k < nwarp; k++) {
+                wpre += k < warp ? s_w[k] : 0;
+                tot += s_w[k];
+            }
+            if (i < G) st_relaxed(&res[i], kSlotFlag | (run + wpre + incl - v));
+            run += tot;
+        }
+    }
+    if (threadIdx.x == 0) {
+        uint64_t v;
+        while (!((v = ld_relaxed(&res[blockIdx.x])) & kSlotFlag)) __nanosleep(32);
+        s_val = v & ~kSlotFlag;
+    }
+    __syncthreads();
+    return s_val;
+}
+
+// Grid barrier: every global write made by any thread of any CTA before the
+// call is visible to every thread after it.  `ctr` must be zero.
+__device__ inline void grid_barrier(uint32_t* ctr) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        atomicAdd(ctr, 1u);
+        while (ld_acquire_u32(ctr) < gridDim.x) __nanosleep(64);
+        __threadfence();
+    }
+    __syncthreads();
+}
+
 }  // namespace szx
