@@ -458,90 +458,57 @@ __device__ inline uint32_t size_block(const T (&xv)[VPL], T mu, int& R, bool pro
     return 1 + (uint32_t)(8 * VPL) + warp_sum(m);
 }
 
-// Write the block payload [R][codes][mid-bytes] into shared memory at dst.
+// Write a block payload with shared-memory OR reductions into a zero-filled
+// staging area: every byte of [R][codes][mid-bytes] is OR-ed into its 32-bit
+// word, so neighbouring values, lanes and blocks may share boundary words
+// without byte stores or run assembly.  dst is the shared-memory address of
+// the block payload; values [0, cnt) of the lane are valid, len in the block.
+__device__ inline void red_or_s(uint32_t a, uint32_t v) {
+    asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ inline void red_or_byte(uint32_t a, uint32_t v) { red_or_s(a & ~3u, (v & 0xFFu) << (8 * (a & 3u))); }
+
 template <typename T, int VPL>
-__device__ inline void pack_block(const typename Traits<T>::U (&u)[VPL], const LaneCode& lc, int cnt, int len,
-                                  uint8_t* dst) {
+__device__ inline void pack_red(const typename Traits<T>::U (&u)[VPL], const LaneCode& lc, int cnt, int len,
+                                uint32_t dst) {
     using TR = Traits<T>;
+    using U = typename TR::U;
     constexpr int W = TR::W;
     const int lane = threadIdx.x & 31;
     const int ncode = (len + 3) / 4;
     const bool raw = lc.R >= TR::kFull;
     const int s = raw ? 0 : ((8 - (lc.R & 7)) & 7);
     const int req = (lc.R + s) >> 3;
-    if (lane == 0) dst[0] = (uint8_t)lc.R;
-    // code bytes: lane l owns bytes [l*VPL/4, (l+1)*VPL/4)  (R8: LSB-first)
+    if (lane == 0) red_or_byte(dst, (uint32_t)lc.R);
 #pragma unroll
     for (int q = 0; q < VPL / 4; q++) {
         const int cb = lane * (VPL / 4) + q;
-        if (cb < ncode) dst[1 + cb] = (uint8_t)(lc.leads >> (8 * q));
+        if (cb < ncode) red_or_byte(dst + 1 + cb, lc.leads >> (8 * q));
     }
-    // mid-bytes: bytes [W-req, W-lead) of each little-endian word (R7).  The
-    // lane's run is assembled in registers (last value first, shifting left)
-    // and written with 32-bit stores; only the partial end words go byte-wise.
-    using U = typename TR::U;
-    constexpr int NW = VPL * W / 4;
-    uint32_t run[NW];
+    uint32_t a = dst + 1 + ncode + lc.mexcl;
 #pragma unroll
-    for (int q = 0; q < NW; q++) run[q] = 0;
-    int rlen = 0;
-#pragma unroll
-    for (int i = VPL - 1; i >= 0; i--) {
-        if (i < cnt) {
-            const int L = (lc.leads >> (2 * i)) & 3;
-            const int mi = req > L ? req - L : 0;
-            run_shl<NW>(run, mi);
-            U bytes = u[i] >> (8 * (W - req));
-            bytes &= mi >= W ? ~U(0) : ((U(1) << (8 * mi)) - U(1));
-            run[0] |= (uint32_t)bytes;
-            if (W == 8) run[1] |= (uint32_t)((uint64_t)bytes >> 32);
-            rlen += mi;
-        }
-    }
-    run_store<NW>(dst + 1 + ncode + lc.mexcl, run, rlen);
-}
-
-// Fast path of pack_block for a FULL block: run assembled with clamped
-// funnel shifts, written with predicated 32-bit / byte shared stores.
-// dst is the shared-memory address of the block payload.
-template <typename T, int VPL>
-__device__ inline void pack_full(const typename Traits<T>::U (&u)[VPL], const LaneCode& lc, uint32_t dst) {
-    using TR = Traits<T>;
-    using U = typename TR::U;
-    constexpr int W = TR::W;
-    constexpr int NCODE = 8 * VPL;
-    constexpr int NW = VPL * W / 4;
-    const int lane = threadIdx.x & 31;
-    const bool raw = lc.R >= TR::kFull;
-    const int s = raw ? 0 : ((8 - (lc.R & 7)) & 7);
-    const int req = (lc.R + s) >> 3;
-    sts_u8_if(lane == 0, dst, (uint32_t)lc.R);
-#pragma unroll
-    for (int q = 0; q < VPL / 4; q++) sts_u8_if(true, dst + 1 + lane * (VPL / 4) + q, lc.leads >> (8 * q));
-    uint32_t run[NW];
-#pragma unroll
-    for (int q = 0; q < NW; q++) run[q] = 0;
-    int rlen = 0;
-#pragma unroll
-    for (int i = VPL - 1; i >= 0; i--) {
+    for (int i = 0; i < VPL; i++) {
         const int L = (lc.leads >> (2 * i)) & 3;
         const int mi = req > L ? req - L : 0;
-        // drop the L lead bytes at the top, then bring the mid-bytes down
-        const U hi = u[i] << (8 * L);
-        const int rs = 8 * (W - req + L);
-        if (W == 4) {
-            run_push4<NW>(run, mi);
-            run[0] |= __funnelshift_rc((uint32_t)hi, 0u, rs);   // clamped: rs >= 32 gives 0
-        } else {
-            run_push4<NW>(run, mi > 4 ? mi - 4 : 0);
-            run_push4<NW>(run, mi < 4 ? mi : 4);
-            const uint64_t bm = rs >= 64 ? 0ull : ((uint64_t)hi >> rs);
-            run[0] |= (uint32_t)bm;
-            run[1] |= (uint32_t)(bm >> 32);
+        if (i < cnt && mi > 0) {
+            // the mid-bytes: bytes [W-req, W-L) of the word, brought down to byte 0
+            const U chunk = (U)(u[i] << (8 * L)) >> (8 * (W - req + L));
+            const uint32_t sh = 8 * (a & 3u), wa = a & ~3u;
+            const uint32_t c0 = (uint32_t)chunk;
+            if (W == 4) {
+                red_or_s(wa, c0 << sh);
+                const uint32_t w1 = __funnelshift_l(c0, 0u, sh);
+                if (w1) red_or_s(wa + 4, w1);
+            } else {
+                const uint32_t c1 = (uint32_t)((uint64_t)chunk >> 32);
+                red_or_s(wa, c0 << sh);
+                const uint32_t w1 = __funnelshift_l(c0, c1, sh), w2 = __funnelshift_l(c1, 0u, sh);
+                if (w1) red_or_s(wa + 4, w1);
+                if (w2) red_or_s(wa + 8, w2);
+            }
+            a += mi;
         }
-        rlen += mi;
     }
-    run_store_s<NW>(dst + 1 + NCODE + lc.mexcl, run, rlen);
 }
 
 // ------------------------------------------------------------------ K2 size pass
@@ -841,8 +808,12 @@ __global__ void __launch_bounds__(256) k_enc_write(const T* __restrict__ x, Plan
     const uint64_t base = p.gbase[t];
     const uint32_t Tb = __shfl_sync(0xffffffffu, zincl, 31);
     const int sb = (int)(base & 15);
+    {   // zero the staging area the OR reductions assemble the tile in
+        const uint32_t nz = (uint32_t)((sb + Tb + 15) >> 4);
+        for (uint32_t ch = threadIdx.x; ch < nz; ch += 256) reinterpret_cast<uint4*>(stg)[ch] = make_uint4(0, 0, 0, 0);
+    }
     cp_async_wait<0>();
-    __syncwarp();
+    __syncthreads();
 #pragma unroll 1
     for (int j = 0; j < C::BPW; j++) {
         const int bi = warp * C::BPW + j;
@@ -860,12 +831,12 @@ __global__ void __launch_bounds__(256) k_enc_write(const T* __restrict__ x, Plan
             for (int q = 0; q < C::QV; q++)
                 reinterpret_cast<uint4*>(xv)[q] = lds_u128(sin + j * C::BW + (lane * C::QV + q) * 16);
             encode_known_R<T, VPL>(xv, VPL, C::B, cmu, R, u, lc);
-            pack_full<T, VPL>(u, lc, smem_u32(stg) + sb + zo);
+            pack_red<T, VPL>(u, lc, VPL, C::B, smem_u32(stg) + sb + zo);
         } else {  // the partial tail block
             const int cnt = load_lane<T, VPL>(x, p.n, k, lane, xv);
             const int len = (int)(p.n - (uint64_t)k * C::B);
             encode_known_R<T, VPL>(xv, cnt, len, cmu, R, u, lc);
-            pack_block<T, VPL>(u, lc, cnt, len, stg + sb + zo);
+            pack_red<T, VPL>(u, lc, cnt, len, smem_u32(stg) + sb + zo);
         }
     }
     __syncthreads();

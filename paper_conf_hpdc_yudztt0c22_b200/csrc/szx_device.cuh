@@ -184,7 +184,7 @@ __device__ inline uint4 lds_u128(uint32_t a) {
 
 // ---------------------------------------------------------------- shared memory
 // Explicit ld.shared (generic pointers into the staging buffers otherwise
-// compile to generic LD.E).  volatile: keeps them after the mbarrier waits.
+// compile to generic LD.E).
 __device__ inline uint32_t lds_u8(uint32_t a) {
     uint32_t v;
     asm volatile("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(a));
@@ -216,51 +216,6 @@ __device__ inline void run_drop4(uint32_t (&a)[NW], uint32_t k) {
     for (int q = 0; q < NW - 1; q++) a[q] = __funnelshift_rc(a[q], a[q + 1], sh);
     a[NW - 1] = __funnelshift_rc(a[NW - 1], 0u, sh);
 }
-// Predicated shared stores (no branch, no divergence bookkeeping).
-__device__ inline void sts_u8_if(bool c, uint32_t a, uint32_t v) {
-    asm volatile("{ .reg .pred p; setp.ne.b32 p, %2, 0; @p st.shared.u8 [%0], %1; }" ::"r"(a), "r"(v), "r"((int)c)
-                 : "memory");
-}
-__device__ inline void sts_u32_if(bool c, uint32_t a, uint32_t v) {
-    asm volatile("{ .reg .pred p; setp.ne.b32 p, %2, 0; @p st.shared.u32 [%0], %1; }" ::"r"(a), "r"(v), "r"((int)c)
-                 : "memory");
-}
-// Store the first len bytes of a run (NW words) at an arbitrary shared
-// address: aligned 32-bit stores for whole words, byte stores for the
-// partial head word and the partial tail word (shared with neighbours).
-template <int NW>
-__device__ inline void run_store_s(uint32_t a, const uint32_t (&r)[NW], int len) {
-    const uint32_t base = a & ~3u;
-    const int h = (int)(a & 3u), e = h + len;
-    const uint32_t sh = 8 * (uint32_t)h;
-    uint32_t w[NW + 1];
-    w[0] = __funnelshift_lc(0u, r[0], sh);
-#pragma unroll
-    for (int q = 1; q < NW; q++) w[q] = __funnelshift_lc(r[q - 1], r[q], sh);
-    w[NW] = __funnelshift_lc(r[NW - 1], 0u, sh);
-    // whole words
-#pragma unroll
-    for (int q = 0; q <= NW; q++) sts_u32_if(4 * q >= h && 4 * q + 4 <= e, base + 4 * q, w[q]);
-    // head word (bytes h..min(4,e)-1) when it is not whole
-#pragma unroll
-    for (int j = 1; j < 4; j++) sts_u8_if(h > 0 && j >= h && j < e, base + j, w[0] >> (8 * j));
-    // tail word qt = e / 4 (bytes 0..e%4-1) unless it is word 0 with a head
-    const int qt = e >> 2;
-    uint32_t wt = w[0];
-#pragma unroll
-    for (int q = 1; q <= NW; q++) wt = q == qt ? w[q] : wt;
-    const bool tail = (e & 3) != 0 && (qt > 0 || h == 0);
-#pragma unroll
-    for (int j = 0; j < 3; j++) sts_u8_if(tail && j < (e & 3), base + 4 * qt + j, wt >> (8 * j));
-}
-// Insert k (0..4) zero bytes at the front of a run.
-template <int NW>
-__device__ inline void run_push4(uint32_t (&a)[NW], uint32_t k) {
-    const uint32_t sh = 8 * k;
-#pragma unroll
-    for (int q = NW - 1; q > 0; q--) a[q] = __funnelshift_lc(a[q - 1], a[q], sh);
-    a[0] = __funnelshift_lc(0u, a[0], sh);
-}
 
 // ---------------------------------------------------------------- byte runs
 // A lane's run of mid-bytes (at most VPL*W bytes) held little-endian in NW
@@ -283,64 +238,6 @@ __device__ inline void run_shr(uint32_t (&a)[NW], int k) {
     for (int q = 0; q < NW - 1; q++) a[q] = __funnelshift_r(a[q], a[q + 1], sh);
     a[NW - 1] = sh ? a[NW - 1] >> sh : a[NW - 1];
 }
-template <int NW>
-__device__ inline void run_shl(uint32_t (&a)[NW], int k) {
-#pragma unroll
-    for (int r = 0; r < 2; r++) {
-        if (k >= 4) {
-#pragma unroll
-            for (int q = NW - 1; q > 0; q--) a[q] = a[q - 1];
-            a[0] = 0;
-            k -= 4;
-        }
-    }
-    const int sh = 8 * k;
-#pragma unroll
-    for (int q = NW - 1; q > 0; q--) a[q] = __funnelshift_l(a[q - 1], a[q], sh);
-    a[0] = sh ? a[0] << sh : a[0];
-}
-// Load NW words of bytes starting at an arbitrary shared-memory byte address.
-template <int NW>
-__device__ inline void run_load(const uint8_t* p, uint32_t (&a)[NW]) {
-    const uintptr_t addr = reinterpret_cast<uintptr_t>(p);
-    const uint32_t* w = reinterpret_cast<const uint32_t*>(addr & ~uintptr_t(3));
-    const int sh = 8 * (int)(addr & 3);
-    uint32_t lo = w[0];
-#pragma unroll
-    for (int q = 0; q < NW; q++) {
-        const uint32_t hi = w[q + 1];
-        a[q] = __funnelshift_r(lo, hi, sh);
-        lo = hi;
-    }
-}
-// Store the first len bytes of a run at an arbitrary shared-memory byte
-// address: whole words with 32-bit stores, the partial head / tail words
-// byte by byte (they may be shared with the neighbouring lanes' runs).
-template <int NW>
-__device__ inline void run_store(uint8_t* p, const uint32_t (&a)[NW], int len) {
-    if (len <= 0) return;
-    const uintptr_t addr = reinterpret_cast<uintptr_t>(p);
-    uint32_t* w = reinterpret_cast<uint32_t*>(addr & ~uintptr_t(3));
-    const int h = (int)(addr & 3), e = h + len;
-    const int sh = 8 * h;
-    uint32_t prev = 0;
-#pragma unroll
-    for (int q = 0; q <= NW; q++) {
-        const uint32_t cur = q < NW ? a[q] : 0u;
-        const uint32_t word = sh ? __funnelshift_l(prev, cur, sh) : cur;
-        prev = cur;
-        const int b0 = 4 * q, b1 = 4 * q + 4;   // bytes of this word: [b0, b1)
-        if (b0 >= e) break;
-        if (b0 >= h && b1 <= e) {
-            w[q] = word;
-        } else {
-            uint8_t* bp = reinterpret_cast<uint8_t*>(w + q);
-#pragma unroll
-            for (int j = 0; j < 4; j++)
-                if (b0 + j >= h && b0 + j < e) bp[j] = (uint8_t)(word >> (8 * j));
-        }
-    }
-}
 
 // ---------------------------------------------------------------- memory
 __device__ inline uint64_t ld_relaxed(const uint64_t* p) {
@@ -359,45 +256,8 @@ __device__ inline uint4 ld_stream16(const void* p) {
     return v;
 }
 
-// ---------------------------------------------------------------- TMA / mbarrier
+// ---------------------------------------------------------------- addresses
 __device__ inline uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
-__device__ inline void mbar_init(uint64_t* bar, uint32_t count) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
-}
-__device__ inline void fence_mbar_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
-__device__ inline void mbar_arrive(uint64_t* bar) {
-    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
-}
-__device__ inline void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
-                 : "memory");
-}
-// raise the expected transaction bytes of the current phase without arriving
-__device__ inline void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
-    asm volatile("mbarrier.expect_tx.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
-}
-__device__ inline void mbar_wait(uint64_t* bar, uint32_t parity) {
-    asm volatile(
-        "{\n .reg .pred P1;\n"
-        "WAIT_%=:\n"
-        " mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
-        " @!P1 bra WAIT_%=;\n}\n" ::"r"(smem_u32(bar)),
-        "r"(parity)
-        : "memory");
-}
-// 1-D TMA bulk copy global -> shared, completion counted on an mbarrier
-// (bytes and both addresses multiples of 16).
-__device__ inline void tma_load_1d(void* smem_dst, const void* gsrc, uint32_t bytes, uint64_t* bar) {
-    asm volatile(
-        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-            smem_u32(smem_dst)),
-        "l"(gsrc), "r"(bytes), "r"(smem_u32(bar))
-        : "memory");
-}
-// named barrier over the first `nthreads` threads (consumer warps only)
-__device__ inline void bar_sync_named(int id, int nthreads) {
-    asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
-}
 
 // Decoupled look-back (single-pass prefix scan, Merrill & Garland) over
 // per-tile aggregates.  Called by all 32 lanes of ONE warp of the tile's CTA;

@@ -10,5 +10,5 @@ timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
    --log-file gpurun_out/launches_bench.csv python bench.py --steps 3 --warmup 1 --no-cpu --no-e2e \
    > gpurun_out/ncu_launch_bench.log 2>&1; echo "ncu launches rc=$?"
 timeout 1500 ncu --set full --clock-control none --import-source on \
-   -k "regex:k_block_stats|k_classify|k_enc_size|k_zscan|k_enc_write|k_index|k_decode" -s 7 -c 7 \
+   -k "regex:k_block_stats|k_classify|k_enc_size|k_zscan|k_enc_write|k_decode" -s 6 -c 6 \
    -o gpurun_out/prof_full -f python scripts/prof_nyx.py > gpurun_out/ncu_full.log 2>&1; echo "ncu full rc=$?"
