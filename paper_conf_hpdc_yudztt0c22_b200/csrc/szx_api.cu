@@ -111,6 +111,25 @@ bool have_device() {
     return n > 0;
 }
 
+// The library's own temporaries (workspaces of the convenience entry points,
+// device buffers of the host entry points) come from the device's default
+// stream-ordered pool.  Keep freed memory in the pool instead of returning it
+// to the driver at every synchronisation, so repeated calls do not pay for
+// mapping hundreds of MB again.
+void keep_pool_memory() {
+    static thread_local int done_dev = -1;
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return; }
+    if (done_dev == dev) return;
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+        uint64_t thr = ~0ull;
+        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+    cudaGetLastError();
+    done_dev = dev;
+}
+
 uint64_t* pinned_u64() {
     static thread_local uint64_t* p = nullptr;
     if (!p && cudaMallocHost(&p, 64) != cudaSuccess) { cudaGetLastError(); p = nullptr; }
@@ -475,6 +494,7 @@ int64_t szx_compress(const void* d_in, szx_dtype_t dt, uint64_t n, szx_ebmode_t 
     cudaStream_t s = static_cast<cudaStream_t>(stream);
     const uint64_t wsb = szx_compress_workspace_bytes(n, dt, b);
     void* ws = nullptr;
+    keep_pool_memory();
     if (cudaMallocAsync(&ws, wsb, s) != cudaSuccess) { cudaGetLastError(); return SZX_ENOMEM; }
     int64_t r = szx_compress_ws(d_in, dt, n, mode, eb, b, d_out, cap, ws, wsb, stream);
     cudaFreeAsync(ws, s);
@@ -551,6 +571,7 @@ int64_t szx_decompress(const void* d_in, uint64_t in_bytes, void* d_out, uint64_
     const uint64_t W = hs[0].dtype ? 8 : 4;
     if (cap < W * total) return SZX_ENOSPC;
     void* ws = nullptr;
+    keep_pool_memory();
     if (cudaMallocAsync(&ws, wsb, s) != cudaSuccess) { cudaGetLastError(); return SZX_ENOMEM; }
     int64_t r = 0;
     for (size_t i = 0; i < hs.size() && r >= 0; i++) {
@@ -569,6 +590,7 @@ int64_t szx_compress_host(const void* h_in, szx_dtype_t dt, uint64_t n, szx_ebmo
     const uint64_t W = wbytes(dt), bound = szx_compress_bound(n, dt, b);
     if (!block_ok(b)) return SZX_EINVAL;
     void *d_in = nullptr, *d_out = nullptr;
+    keep_pool_memory();
     if (cudaMallocAsync(&d_in, W * n + 16, s) != cudaSuccess) { cudaGetLastError(); return SZX_ENOMEM; }
     if (cudaMallocAsync(&d_out, bound, s) != cudaSuccess) { cudaGetLastError(); cudaFreeAsync(d_in, s); return SZX_ENOMEM; }
     int64_t r = SZX_ECUDA;
@@ -589,6 +611,7 @@ int64_t szx_decompress_host(const void* h_in, uint64_t in_bytes, void* h_out, ui
     if (!have_device()) return SZX_ECUDA;
     cudaStream_t s = static_cast<cudaStream_t>(stream);
     void* d_in = nullptr;
+    keep_pool_memory();
     if (cudaMallocAsync(&d_in, in_bytes, s) != cudaSuccess) { cudaGetLastError(); return SZX_ENOMEM; }
     int64_t r = SZX_ECUDA;
     if (cudaMemcpyAsync(d_in, h_in, in_bytes, cudaMemcpyHostToDevice, s) == cudaSuccess) {
