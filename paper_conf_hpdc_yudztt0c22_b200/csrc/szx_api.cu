@@ -336,14 +336,15 @@ constexpr uint64_t kMaxDecodeGrid = 2048;  // co-resident CTAs of k_decode_w (sl
 
 struct DLayout {
     uint64_t nB, nW;
-    uint64_t zero_bytes, off_ncpre, off_tbase, total;
+    uint64_t zero_bytes, off_nctile, off_ncpre, off_tbase, total;
 };
 DLayout dlayout(uint64_t n, uint32_t b) {
     DLayout L{};
     L.nB = cdiv(n, b);
     L.nW = cdiv(L.nB, 32);
-    L.zero_bytes = 16 + 16 + 4 * 8 * kMaxDecodeGrid;  // ctr[4], err, slot_a, res_a, slot_z, res_z
-    L.off_ncpre = L.zero_bytes;
+    L.zero_bytes = 32 + 16 + 16 + 4 * 8 * kMaxDecodeGrid;  // ctr[8], err, n_nctile, slot_a, res_a, slot_z, res_z
+    L.off_nctile = L.zero_bytes;
+    L.off_ncpre = al16(L.off_nctile + 4 * L.nW);
     L.off_tbase = al16(L.off_ncpre + 4 * L.nW + 4);
     L.total = al16(L.off_tbase + 8 * (L.nW + 1)) + 256;
     return L;
@@ -394,11 +395,13 @@ int enqueue_decompress(const void* d_in, uint64_t in_bytes, const szx_header_t* 
     p.b = h->block_size;
     p.dtype = h->dtype;
     p.ctr = reinterpret_cast<uint32_t*>(ws);
-    p.err = reinterpret_cast<int32_t*>(ws + 16);
-    p.slot_a = reinterpret_cast<uint64_t*>(ws + 32);
+    p.err = reinterpret_cast<int32_t*>(ws + 32);
+    p.n_nctile = reinterpret_cast<uint32_t*>(ws + 48);
+    p.slot_a = reinterpret_cast<uint64_t*>(ws + 64);
     p.res_a = p.slot_a + kMaxDecodeGrid;
     p.slot_z = p.res_a + kMaxDecodeGrid;
     p.res_z = p.slot_z + kMaxDecodeGrid;
+    p.nctile = reinterpret_cast<uint32_t*>(ws + L.off_nctile);
     p.ncpre = reinterpret_cast<uint32_t*>(ws + L.off_ncpre);
     p.tbase = reinterpret_cast<uint64_t*>(ws + L.off_tbase);
     *d_err_out = p.err;

@@ -31,11 +31,13 @@ struct DPlan {
     uint64_t n, nB, nW, in_bytes;
     uint64_t off_mu;
     uint32_t b, dtype;
-    uint32_t* ctr;             // [4] init 0: [0] [3] prefix arrivals, [1] tile counter, [2] grid barrier
+    uint32_t* ctr;             // [8] init 0: [0] [3] prefix arrivals, [1] [4] tile counters, [2] grid barrier
     uint64_t* slot_a;          // [grid] per-CTA nonconstant counts
     uint64_t* res_a;           // [grid] init 0: their exclusive prefixes
     uint64_t* slot_z;          // [grid] per-CTA payload byte counts
     uint64_t* res_z;           // [grid] init 0: their exclusive prefixes
+    uint32_t* nctile;          // [nW]      tiles holding nonconstant blocks (+ a partial last tile)
+    uint32_t* n_nctile;        // [1]       their count
     uint32_t* ncpre;           // [nW]      nonconstant index of each tile's first block
     uint64_t* tbase;           // [nW + 1]  payload offset of each tile (tbase[nW] = total)
     int32_t* err;              // 0 ok, else SZX_ECORRUPT
@@ -142,13 +144,21 @@ __device__ inline void index_phase(const DPlan& p, const uint8_t* __restrict__ i
         if (w == p.nW - 1 && (p.nB & 31)) x &= (1u << (p.nB & 31)) - 1u;  // ignore padding bits
         return x;
     };
-    // (1) nonconstant blocks in the range -> starting nonconstant index
+    // tiles the nonconstant warps visit: those with nonconstant blocks, and a
+    // partial last tile (it is decoded whole by the generic path)
+    const uint64_t nW_full = p.n / ((uint64_t)kTileBlocks * 32 * (p.b / 32));
+    auto nc_tile = [&](uint64_t w, uint32_t word) -> uint64_t { return (word != 0u || w >= nW_full) ? 1u : 0u; };
+    // (1) nonconstant blocks (low 32 bits) and such tiles (high 32 bits) in the
+    // range -> starting nonconstant index and list position.  nNC <= 2^29.
     uint64_t cnt = 0;
-    for (uint64_t w = w0 + threadIdx.x; w < w1; w += kIndexChunk) cnt += __popc(word_at(w));
-    const uint64_t aggA = cta_sum64(cnt, s_w);
-    if (SZX_EXP & 128) { if (threadIdx.x == 0 && aggA == 12345) p.ncpre[0] = 1; return; }
-    const uint64_t exA = grid_excl_prefix(p.slot_a, p.res_a, &p.ctr[0], aggA, s_w);
-    if (SZX_EXP & 64) { if (threadIdx.x == 0 && exA == 12345) p.ncpre[0] = 1; return; }
+    for (uint64_t w = w0 + threadIdx.x; w < w1; w += kIndexChunk) {
+        const uint32_t x = word_at(w);
+        cnt += __popc(x) | (nc_tile(w, x) << 32);
+    }
+    const uint64_t aggP = cta_sum64(cnt, s_w);
+    const uint64_t exP = grid_excl_prefix(p.slot_a, p.res_a, &p.ctr[0], aggP, s_w);
+    const uint64_t aggA = aggP & 0xFFFFFFFFu, exA = exP & 0xFFFFFFFFu;
+    uint64_t runT = exP >> 32;
     const bool ok = exA + aggA <= hd.nnc;
     // (2) their payload bytes -> starting payload offset.  A range of at most
     // one chunk keeps its zsizes in shared memory for step (3).
@@ -171,9 +181,15 @@ __device__ inline void index_phase(const DPlan& p, const uint8_t* __restrict__ i
         const uint64_t w = wc + threadIdx.x;
         const uint32_t word = w < w1 ? word_at(w) : 0u;
         const uint32_t cw = __popc(word);
-        uint64_t tot;
-        const uint64_t ex = cta_scan256(cw, &tot, s_w);
-        if (w < w1) p.ncpre[w] = (uint32_t)(runA + ex);
+        const uint64_t isnc = w < w1 ? nc_tile(w, word) : 0u;
+        uint64_t totP;
+        const uint64_t exq = cta_scan256(cw | (isnc << 32), &totP, s_w);
+        const uint64_t ex = exq & 0xFFFFFFFFu, tot = totP & 0xFFFFFFFFu;
+        if (w < w1) {
+            p.ncpre[w] = (uint32_t)(runA + ex);
+            if (isnc) p.nctile[runT + (exq >> 32)] = (uint32_t)w;
+        }
+        runT += totP >> 32;
         if (!one) {
             if (ok) stage_u16(s_zs, zs, runA, tot);
             __syncthreads();
@@ -192,6 +208,7 @@ __device__ inline void index_phase(const DPlan& p, const uint8_t* __restrict__ i
         if (!ok) set_corrupt(p.err);
         if (c == G - 1) {
             p.tbase[p.nW] = runZ;
+            *p.n_nctile = (uint32_t)runT;
             if (runA != hd.nnc || runZ != hd.payload_bytes) set_corrupt(p.err);
         }
     }
@@ -431,6 +448,16 @@ struct DecWCfg {
     static constexpr int NT = 256, NWARP = NT / 32;
     static constexpr int SLOT = SZX_DSLOT;          // tile payload bytes staged in shared memory
     static constexpr int SLOT_ALLOC = SLOT + 64;    // + over-read pad of the last block's run loads
+#ifndef SZX_FILLW
+#define SZX_FILLW 2
+#endif
+#ifndef SZX_FSTATIC
+#define SZX_FSTATIC 0
+#endif
+#ifndef SZX_SWITCH
+#define SZX_SWITCH 2
+#endif
+    static constexpr int FILLW = SZX_FILLW;         // fill warps per CTA (the rest decode)
     static constexpr int SMEM = NWARP * 2 * SLOT_ALLOC;
     static_assert(SMEM >= kIndexChunk * 32 * 2, "index-phase scratch aliases the slots");
 };
@@ -480,6 +507,51 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
     const uint64_t nW_full = p.n / ((uint64_t)TB * B);
     const uint32_t slot0 = smem_u32(dsm + (threadIdx.x >> 5) * 2 * C::SLOT_ALLOC);
 
+    // ---- fill warps: the constant blocks of every full tile (Fig. 10 state 0:
+    // retrieve with mu).  They need only the bitmap word and the tile's mu
+    // values, prefetched one tile ahead, so they stream stores.
+    auto fill_loop = [&]() {
+#if SZX_FSTATIC
+        uint64_t fnext = ((uint64_t)blockIdx.x * C::FILLW + (threadIdx.x >> 5));
+        auto grab_f = [&]() -> uint64_t {
+            const uint64_t v = fnext;
+            fnext += (uint64_t)gridDim.x * C::FILLW;
+            return v;
+        };
+#else
+        auto grab_f = [&]() -> uint64_t {
+            uint32_t v = 0;
+            if (lane == 0) v = atomicAdd(&p.ctr[1], 1u);
+            return __shfl_sync(0xffffffffu, v, 0);
+        };
+#endif
+        uint64_t t = grab_f();
+        uint32_t word = 0;
+        U mul = 0;
+        if (t < nW_full) { word = bm[t]; mul = mus[t * TB + lane]; }
+        while (t < nW_full) {
+            const uint64_t tn = grab_f();
+            uint32_t wn = 0;
+            U mn = 0;
+            if (tn < nW_full) { wn = bm[tn]; mn = mus[tn * TB + lane]; }
+            uint4* yq = reinterpret_cast<uint4*>(y + t * TB * B + lane * VPL);
+#pragma unroll 2
+            for (uint32_t m = ~word; m; m &= m - 1) {
+                const int j = __ffs(m) - 1;
+                const U mb = __shfl_sync(0xffffffffu, mul, j);
+                T v[VPL];
+#pragma unroll
+                for (int q = 0; q < VPL; q++) v[q] = TR::from(mb);
+#pragma unroll
+                for (int q = 0; q < NV; q++) st_out16(yq + j * QB + q, reinterpret_cast<const uint4*>(v)[q]);
+            }
+            t = tn;
+            word = wn;
+            mul = mn;
+        }
+    };
+    const uint32_t n_nct = *p.n_nctile;
+
     auto load_meta = [&](uint64_t t, TileMeta<U>& m) {
         uint32_t word = bm[t];
         if (t == p.nW - 1 && (p.nB & 31)) word &= (1u << (p.nB & 31)) - 1u;
@@ -512,12 +584,19 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
     };
     // dynamic tile assignment: nonconstant-heavy tiles cost far more than
     // constant ones, so static striding leaves warps idle at the end
+    // nonconstant warps: dynamic assignment over the list of tiles holding
+    // nonconstant blocks (their cost varies far more than the fill's)
     auto grab = [&]() -> uint64_t {
-        uint32_t v = 0;
-        if (lane == 0) v = atomicAdd(&p.ctr[1], 1u);
-        return __shfl_sync(0xffffffffu, v, 0);
+        uint32_t v = 0xFFFFFFFFu;
+        if (lane == 0) {
+            const uint32_t i = atomicAdd(&p.ctr[4], 1u);
+            if (i < n_nct) v = p.nctile[i];
+        }
+        v = __shfl_sync(0xffffffffu, v, 0);
+        return v == 0xFFFFFFFFu ? p.nW : (uint64_t)v;
     };
 
+    auto nc_loop = [&]() {
     uint64_t t = grab();
     if (t >= p.nW) return;
     TileMeta<U> cur, nx;
@@ -540,29 +619,6 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
         const uint32_t zoff = zincl - zl;
         const uint64_t k0 = t * TB;
         const bool full = t < nW_full;
-        // constant blocks of a full tile: retrieve with mu (Fig. 10, state 0)
-        if (ok && full && !(SZX_EXP & 1)) {
-            uint4* yq = reinterpret_cast<uint4*>(y + k0 * B + lane * VPL);
-#pragma unroll 2
-#if SZX_ROT
-            // start each tile at a different block so that concurrently active
-            // warps spread their stores over the address space
-            const uint32_t rot = (uint32_t)(t * 13) & 31u;
-            const uint32_t cw = (SZX_EXP & 4) ? ~0u : ~word;
-            for (uint32_t m = __funnelshift_r(cw, cw, rot); m; m &= m - 1) {
-                const int j = (__ffs(m) - 1 + rot) & 31;
-#else
-            for (uint32_t m = (SZX_EXP & 4) ? ~0u : ~word; m; m &= m - 1) {
-                const int j = __ffs(m) - 1;
-#endif
-                const U mb = __shfl_sync(0xffffffffu, cur.mul, j);
-                T v[VPL];
-#pragma unroll
-                for (int q = 0; q < VPL; q++) v[q] = TR::from(mb);
-#pragma unroll
-                for (int q = 0; q < NV; q++) st_out16(yq + j * QB + q, reinterpret_cast<const uint4*>(v)[q]);
-            }
-        }
         // prefetch the next tile's payload into the other slot
         uint32_t nx_staged = 0;
         if (tn < p.nW) {
@@ -631,6 +687,20 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
         t = tn;
     }
     cp_async_wait<0>();
+    };
+    // Each warp drains its own queue first, then helps with the other one, so
+    // the split adapts to the field's fraction of nonconstant blocks.
+    if (SZX_EXP & 256) {
+        if ((int)(threadIdx.x >> 5) < C::FILLW) fill_loop();
+        return;
+    }
+    if ((int)(threadIdx.x >> 5) < C::FILLW) {
+        fill_loop();
+        if (SZX_SWITCH & 2) nc_loop();
+    } else {
+        nc_loop();
+        if (SZX_SWITCH & 1) fill_loop();
+    }
 }
 
 }  // namespace szx
