@@ -326,7 +326,6 @@ def main():
             "k_enc_size": nnc * 128 * 4 + 2 * nnc + 5 * nnc,
             "k_zscan": 2 * nnc,
             "k_enc_write": nnc * 128 * 4 + 5 * nnc + pb,
-            "k_index": nB // 8 + 2 * nnc,
             "k_decode": S + nbytes,
         }
         dom = max(kms, key=lambda k: kms[k]) if kms else None
