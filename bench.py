@@ -121,8 +121,9 @@ def _ncu_traffic(kernel: str):
     if not files:
         return None, None
     d = json.load(open(files[-1]))
+    ncu_name = {"k_decode": "k_decode_w"}.get(kernel, kernel)  # timing label -> template name
     for name, v in d.items():
-        if name.startswith(kernel + "<") or name == kernel:
+        if name.startswith(ncu_name + "<") or name == ncu_name:
             return v.get("dram_bytes"), os.path.basename(files[-1])
     return None, None
 

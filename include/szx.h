@@ -117,6 +117,27 @@ int szx_read_header(const void* h_bytes, uint64_t nbytes, szx_header_t* out);
 int64_t szx_decompress(const void* d_in, uint64_t in_bytes, void* d_out,
                        uint64_t out_capacity_bytes, void* stream);
 
+/* Decompress only blocks [first_block, first_block + n_blocks) of a stream
+ * (SZX1) or container (SZXC), the "1 stream -> Q GPUs" path of SURVEY 8(e):
+ * each rank decodes its own block range.  The decoder still reads the bitmap
+ * and zsize sections up to the range (the paper's prefix sum over block
+ * sizes; <= 0.42 % of the raw size for f32, b = 128) and
+ * decodes only the tiles of the range (Fig. 10's five steps).
+ *   first_block  global block index (blocks of the stream's block_size; in a
+ *                container, blocks are numbered over the whole array, and
+ *                every shard must start on a block boundary -- true for
+ *                block-range shards -- else SZX_EINVAL);
+ *   n_blocks     count, clipped to the end of the array;
+ *   d_out        device, >= 16-byte aligned; receives values
+ *                [first_block * b, min(n, (first_block + n_blocks) * b)),
+ *                element 0 being the first value of first_block;
+ *   out_capacity_bytes >= that count * W, else SZX_ENOSPC.
+ * Blocking (reads headers and the status back).  Returns the number of
+ * values written (0 for an empty range), or SZX_EINVAL / SZX_ECORRUPT /
+ * SZX_ECUDA / SZX_ENOMEM.  Output equals the same slice of szx_decompress. */
+int64_t szx_decompress_blocks(const void* d_in, uint64_t in_bytes, uint64_t first_block, uint64_t n_blocks,
+                              void* d_out, uint64_t out_capacity_bytes, void* stream);
+
 /* As szx_decompress (SZX1 only) with a caller workspace. */
 int64_t szx_decompress_ws(const void* d_in, uint64_t in_bytes, void* d_out,
                           uint64_t out_capacity_bytes, void* d_ws, uint64_t ws_bytes, void* stream);

@@ -376,20 +376,30 @@ int parse_header(const uint8_t* b, uint64_t nbytes, szx_header_t* h) {
 
 // Only h->n, h->dtype and h->block_size are used on the host; the kernels
 // read and validate the content-dependent header fields on the device.
+// Reconstructs blocks [kb0, kb1) (kb1 = UINT64_MAX: to the end) into d_out,
+// whose element 0 is the first value of block kb0.
 int enqueue_decompress(const void* d_in, uint64_t in_bytes, const szx_header_t* h, void* d_out,
-                       uint64_t cap, void* d_ws, uint64_t ws_bytes, int32_t** d_err_out, cudaStream_t s) {
+                       uint64_t cap, void* d_ws, uint64_t ws_bytes, int32_t** d_err_out, cudaStream_t s,
+                       uint64_t kb0 = 0, uint64_t kb1 = UINT64_MAX) {
     if (!d_in || !aligned16(d_in) || !h) return SZX_EINVAL;
     if (h->dtype > 1 || !block_ok(h->block_size) || h->n > kMaxN) return SZX_EINVAL;
     if (in_bytes < kHeaderBytes) return SZX_ECORRUPT;
     const uint64_t W = h->dtype ? 8 : 4;
-    if (cap < W * h->n) return SZX_ENOSPC;
-    if (h->n && (!d_out || !aligned16(d_out))) return SZX_EINVAL;
+    const uint64_t nBh = cdiv(h->n, h->block_size);
+    if (kb1 > nBh) kb1 = nBh;
+    if (kb0 > kb1) return SZX_EINVAL;
+    const uint64_t e0 = kb0 * h->block_size, e1 = std::min<uint64_t>(h->n, kb1 * h->block_size);
+    const uint64_t n_out = e1 - e0;
+    if (cap < W * n_out) return SZX_ENOSPC;
+    if (n_out && (!d_out || !aligned16(d_out))) return SZX_EINVAL;
     DLayout L = dlayout(h->n, h->block_size);
     if (!d_ws || !aligned16(d_ws)) return SZX_EINVAL;
     if (ws_bytes < L.total) return SZX_ENOSPC;
     uint8_t* ws = static_cast<uint8_t*>(d_ws);
     DPlan p{};
     p.n = h->n; p.nB = L.nB; p.nW = L.nW;
+    p.kb0 = kb0; p.kb1 = kb1;
+    p.nWi = cdiv(kb1, 32); p.t_lo = kb0 / 32;
     p.in_bytes = in_bytes;
     p.off_mu = kHeaderBytes + al16(cdiv(L.nB, 8));
     p.b = h->block_size;
@@ -406,8 +416,11 @@ int enqueue_decompress(const void* d_in, uint64_t in_bytes, const szx_header_t* 
     p.tbase = reinterpret_cast<uint64_t*>(ws + L.off_tbase);
     *d_err_out = p.err;
     cudaMemsetAsync(ws, 0, L.zero_bytes, s);
-    if (h->n == 0) return cudaGetLastError() == cudaSuccess ? SZX_OK : SZX_ECUDA;
+    if (n_out == 0) return cudaGetLastError() == cudaSuccess ? SZX_OK : SZX_ECUDA;
     const uint8_t* in = static_cast<const uint8_t*>(d_in);
+    // the kernels index the output by stream element; shift the base so that
+    // element e0 lands on d_out[0] (only elements of [e0, e1) are stored)
+    const uintptr_t ybase = reinterpret_cast<uintptr_t>(d_out) - W * e0;
     dispatch((szx_dtype_t)h->dtype, h->block_size, [&](auto tag, auto vpl) {
         using T = decltype(tag);
         constexpr int V = decltype(vpl)::value;
@@ -420,12 +433,13 @@ int enqueue_decompress(const void* d_in, uint64_t in_bytes, const szx_header_t* 
             cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_decode_w<T, V>, 256, DecWCfg<T, V>::SMEM);
             if (occ <= 0) occ = 4;
         }
-        uint64_t grid = cdiv(L.nW, 8);
+        uint64_t grid = cdiv(p.nWi, 8);
         const uint64_t cap = (uint64_t)sm_count() * occ;
         if (grid > cap) grid = cap;
         if (grid > kMaxDecodeGrid) grid = kMaxDecodeGrid;
         launch("k_decode", s, [&] {
-            launch_pdl(k_decode_w<T, V>, dim3((unsigned)grid), dim3(256), DecWCfg<T, V>::SMEM, s, p, in, static_cast<T*>(d_out));
+            launch_pdl(k_decode_w<T, V>, dim3((unsigned)grid), dim3(256), DecWCfg<T, V>::SMEM, s, p, in,
+                       reinterpret_cast<T*>(ybase));
         });
     });
     return cudaGetLastError() == cudaSuccess ? SZX_OK : SZX_ECUDA;
@@ -446,6 +460,123 @@ int64_t decompress_one_sync(const void* d_in, uint64_t in_bytes, const szx_heade
     if (read_device_bytes(d_err, &err, 4, s)) return SZX_ECUDA;
     timing_resolve();
     return err ? err : (int64_t)h->n;
+}
+
+// ------------------------------------------------------------ stream sets
+// An SZX1 stream is one part; an SZXC container (DESIGN.md s.4) is P parts,
+// part i holding elements [first_i, first_i + n_i) of the array.
+struct Part {
+    szx_header_t h;
+    uint64_t off, len, first;
+};
+
+int parse_parts(const void* d_in, uint64_t in_bytes, cudaStream_t s, std::vector<Part>& parts, uint64_t* total) {
+    uint8_t hb[64];
+    if (read_device_bytes(d_in, hb, 64, s)) return SZX_ECUDA;
+    parts.clear();
+    if (memcmp(hb, "SZXC", 4) == 0) {
+        uint32_t P, ver;
+        uint64_t total_n;
+        memcpy(&ver, hb + 4, 4);
+        memcpy(&P, hb + 8, 4);
+        memcpy(&total_n, hb + 16, 8);
+        if (ver != 1 || P == 0 || 32 + 32ull * P > in_bytes) return SZX_ECORRUPT;
+        std::vector<uint8_t> tab(32ull * P);
+        if (read_device_bytes(static_cast<const uint8_t*>(d_in) + 32, tab.data(), tab.size(), s)) return SZX_ECUDA;
+        uint64_t expect = 0;
+        for (uint32_t i = 0; i < P; i++) {
+            uint64_t e[4];
+            memcpy(e, tab.data() + 32ull * i, 32);
+            if (e[0] != expect || e[2] % 16 || e[2] > in_bytes || e[3] > in_bytes - e[2] || e[3] < 64)
+                return SZX_ECORRUPT;
+            uint8_t sh[64];
+            if (read_device_bytes(static_cast<const uint8_t*>(d_in) + e[2], sh, 64, s)) return SZX_ECUDA;
+            Part pt;
+            if (parse_header(sh, 64, &pt.h) || pt.h.n != e[1]) return SZX_ECORRUPT;
+            if (!parts.empty() && pt.h.dtype != parts[0].h.dtype) return SZX_ECORRUPT;
+            pt.off = e[2]; pt.len = e[3]; pt.first = e[0];
+            parts.push_back(pt);
+            expect += e[1];
+        }
+        if (expect != total_n) return SZX_ECORRUPT;
+        *total = total_n;
+    } else {
+        Part pt;
+        if (parse_header(hb, 64, &pt.h)) return SZX_ECORRUPT;
+        pt.off = 0; pt.len = in_bytes; pt.first = 0;
+        parts.push_back(pt);
+        *total = pt.h.n;
+    }
+    return SZX_OK;
+}
+
+// Decode global blocks [g0, g1) of a stream or container into d_out (element
+// 0 = first value of block g0).  Every part's kernel is enqueued back to back
+// (each with its own workspace slice), then one synchronisation reads all
+// status words.  ranged: block indices are global over the container, which
+// requires every part to start on a block boundary of one common block size.
+int64_t decode_range(const void* d_in, uint64_t in_bytes, uint64_t g0, uint64_t g1, void* d_out, uint64_t cap,
+                     cudaStream_t s, bool ranged) {
+    if (!d_in || in_bytes < 64) return SZX_ECORRUPT;
+    if (!have_device()) return SZX_ECUDA;
+    std::vector<Part> parts;
+    uint64_t total = 0;
+    int rc = parse_parts(d_in, in_bytes, s, parts, &total);
+    if (rc) return rc;
+    const uint64_t W = parts[0].h.dtype ? 8 : 4;
+    const uint64_t b = parts[0].h.block_size;
+    if (ranged)
+        for (auto& pt : parts)
+            if (pt.h.block_size != b || pt.first % b) return SZX_EINVAL;
+    const uint64_t nBg = cdiv(total, b);
+    if (g1 > nBg) g1 = nBg;
+    if (g0 > g1) g0 = g1;  // a range starting past the end is empty
+    const uint64_t e0 = ranged ? g0 * b : 0, e1 = ranged ? std::min(total, g1 * b) : total;
+    const uint64_t n_out = e1 > e0 ? e1 - e0 : 0;
+    if (cap < W * n_out) return SZX_ENOSPC;
+    if (n_out == 0) return 0;
+    // per part: local block range, output position, workspace slice
+    struct Job { size_t i; uint64_t kb0, kb1, out_el, ws_off; };
+    std::vector<Job> jobs;
+    uint64_t wsb = 0;
+    for (size_t i = 0; i < parts.size(); i++) {
+        const Part& pt = parts[i];
+        const uint64_t pb = pt.h.block_size, nBp = cdiv(pt.h.n, pb);
+        uint64_t kb0 = 0, kb1 = nBp;
+        if (ranged) {
+            const uint64_t f = pt.first / b;
+            if (f + nBp <= g0 || f >= g1) continue;
+            kb0 = g0 > f ? g0 - f : 0;
+            kb1 = std::min(nBp, g1 - f);
+        }
+        if (pt.h.n == 0) continue;
+        jobs.push_back({i, kb0, kb1, pt.first + kb0 * pb - e0, wsb});
+        wsb += al16(szx_decompress_workspace_bytes(&pt.h));
+    }
+    void* ws = nullptr;
+    keep_pool_memory();
+    if (cudaMallocAsync(&ws, std::max<uint64_t>(wsb, 16), s) != cudaSuccess) { cudaGetLastError(); return SZX_ENOMEM; }
+    std::vector<int32_t*> errs;
+    int64_t r = 0;
+    for (const Job& j : jobs) {
+        const Part& pt = parts[j.i];
+        int32_t* d_err = nullptr;
+        const uint64_t wsz = al16(szx_decompress_workspace_bytes(&pt.h));
+        rc = enqueue_decompress(static_cast<const uint8_t*>(d_in) + pt.off, pt.len, &pt.h,
+                                static_cast<uint8_t*>(d_out) + W * j.out_el, cap - W * j.out_el,
+                                static_cast<uint8_t*>(ws) + j.ws_off, wsz, &d_err, s, j.kb0, j.kb1);
+        if (rc) { r = rc; break; }
+        errs.push_back(d_err);
+    }
+    if (r == 0 && cudaStreamSynchronize(s) != cudaSuccess) r = SZX_ECUDA;
+    for (size_t i = 0; i < errs.size() && r == 0; i++) {
+        int32_t e = 0;
+        if (cudaMemcpy(&e, errs[i], 4, cudaMemcpyDeviceToHost) != cudaSuccess) r = SZX_ECUDA;
+        else if (e) r = e;
+    }
+    timing_resolve();
+    cudaFreeAsync(ws, s);
+    return r < 0 ? r : (int64_t)n_out;
 }
 
 }  // namespace
@@ -533,56 +664,13 @@ int64_t szx_decompress_ws(const void* d_in, uint64_t in_bytes, void* d_out, uint
 }
 
 int64_t szx_decompress(const void* d_in, uint64_t in_bytes, void* d_out, uint64_t cap, void* stream) {
-    if (!d_in || in_bytes < 64) return SZX_ECORRUPT;
-    if (!have_device()) return SZX_ECUDA;
-    cudaStream_t s = static_cast<cudaStream_t>(stream);
-    uint8_t hb[64];
-    if (read_device_bytes(d_in, hb, 64, s)) return SZX_ECUDA;
-    std::vector<szx_header_t> hs;
-    std::vector<uint64_t> offs, lens, firsts;
-    if (memcmp(hb, "SZXC", 4) == 0) {
-        uint32_t P;
-        memcpy(&P, hb + 8, 4);
-        uint32_t ver;
-        memcpy(&ver, hb + 4, 4);
-        uint64_t total_n;
-        memcpy(&total_n, hb + 16, 8);
-        if (ver != 1 || P == 0 || 32 + 32ull * P > in_bytes) return SZX_ECORRUPT;
-        std::vector<uint8_t> tab(32ull * P);
-        if (read_device_bytes(static_cast<const uint8_t*>(d_in) + 32, tab.data(), tab.size(), s)) return SZX_ECUDA;
-        uint64_t expect = 0;
-        for (uint32_t i = 0; i < P; i++) {
-            uint64_t e[4];
-            memcpy(e, tab.data() + 32ull * i, 32);
-            if (e[0] != expect || e[2] % 16 || e[2] + e[3] > in_bytes || e[3] < 64) return SZX_ECORRUPT;
-            uint8_t sh[64];
-            if (read_device_bytes(static_cast<const uint8_t*>(d_in) + e[2], sh, 64, s)) return SZX_ECUDA;
-            szx_header_t h;
-            if (parse_header(sh, 64, &h) || h.n != e[1]) return SZX_ECORRUPT;
-            if (!hs.empty() && h.dtype != hs[0].dtype) return SZX_ECORRUPT;
-            hs.push_back(h); offs.push_back(e[2]); lens.push_back(e[3]); firsts.push_back(e[0]);
-            expect += e[1];
-        }
-        if (expect != total_n) return SZX_ECORRUPT;
-    } else {
-        szx_header_t h;
-        if (parse_header(hb, 64, &h)) return SZX_ECORRUPT;
-        hs.push_back(h); offs.push_back(0); lens.push_back(in_bytes); firsts.push_back(0);
-    }
-    uint64_t wsb = 0, total = 0;
-    for (auto& h : hs) { wsb = std::max<uint64_t>(wsb, szx_decompress_workspace_bytes(&h)); total += h.n; }
-    const uint64_t W = hs[0].dtype ? 8 : 4;
-    if (cap < W * total) return SZX_ENOSPC;
-    void* ws = nullptr;
-    keep_pool_memory();
-    if (cudaMallocAsync(&ws, wsb, s) != cudaSuccess) { cudaGetLastError(); return SZX_ENOMEM; }
-    int64_t r = 0;
-    for (size_t i = 0; i < hs.size() && r >= 0; i++) {
-        r = decompress_one_sync(static_cast<const uint8_t*>(d_in) + offs[i], lens[i], &hs[i],
-                                static_cast<uint8_t*>(d_out) + W * firsts[i], cap - W * firsts[i], ws, wsb, s);
-    }
-    cudaFreeAsync(ws, s);
-    return r < 0 ? r : (int64_t)total;
+    return decode_range(d_in, in_bytes, 0, UINT64_MAX, d_out, cap, static_cast<cudaStream_t>(stream), false);
+}
+
+int64_t szx_decompress_blocks(const void* d_in, uint64_t in_bytes, uint64_t first_block, uint64_t n_blocks,
+                              void* d_out, uint64_t cap, void* stream) {
+    const uint64_t end = n_blocks > UINT64_MAX - first_block ? UINT64_MAX : first_block + n_blocks;
+    return decode_range(d_in, in_bytes, first_block, end, d_out, cap, static_cast<cudaStream_t>(stream), true);
 }
 
 int64_t szx_compress_host(const void* h_in, szx_dtype_t dt, uint64_t n, szx_ebmode_t mode, double eb,

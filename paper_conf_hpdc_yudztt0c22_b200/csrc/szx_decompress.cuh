@@ -30,6 +30,10 @@ struct DPlan {
     // compressed content (nNC, payload size) is read from the header on the device
     uint64_t n, nB, nW, in_bytes;
     uint64_t off_mu;
+    // block range to reconstruct, [kb0, kb1) (whole stream: 0, nB).  The index
+    // phase covers tiles [0, nWi), nWi = ceil(kb1 / 32); only tiles >= t_lo =
+    // kb0 / 32 are decoded; y points at the (virtual) element 0 of the stream.
+    uint64_t kb0, kb1, nWi, t_lo;
     uint32_t b, dtype;
     uint32_t* ctr;             // [8] init 0: [0] [3] prefix arrivals, [1] [4] tile counters, [2] grid barrier
     uint64_t* slot_a;          // [grid] per-CTA nonconstant counts
@@ -136,7 +140,7 @@ template <int W>
 __device__ inline void index_phase(const DPlan& p, const uint8_t* __restrict__ in, const DHdr& hd,
                                    uint16_t* s_zs, uint64_t* s_w) {
     const uint64_t G = gridDim.x, c = blockIdx.x;
-    const uint64_t w0 = p.nW * c / G, w1 = p.nW * (c + 1) / G;
+    const uint64_t w0 = p.nWi * c / G, w1 = p.nWi * (c + 1) / G;
     const uint32_t* bm = reinterpret_cast<const uint32_t*>(in + kHeaderBytes);
     const uint16_t* zs = reinterpret_cast<const uint16_t*>(in + hd.off_zs);
     auto word_at = [&](uint64_t w) -> uint32_t {
@@ -147,7 +151,9 @@ __device__ inline void index_phase(const DPlan& p, const uint8_t* __restrict__ i
     // tiles the nonconstant warps visit: those with nonconstant blocks, and a
     // partial last tile (it is decoded whole by the generic path)
     const uint64_t nW_full = p.n / ((uint64_t)kTileBlocks * 32 * (p.b / 32));
-    auto nc_tile = [&](uint64_t w, uint32_t word) -> uint64_t { return (word != 0u || w >= nW_full) ? 1u : 0u; };
+    auto nc_tile = [&](uint64_t w, uint32_t word) -> uint64_t {
+        return ((word != 0u || w >= nW_full) && w >= p.t_lo) ? 1u : 0u;
+    };
     // (1) nonconstant blocks (low 32 bits) and such tiles (high 32 bits) in the
     // range -> starting nonconstant index and list position.  nNC <= 2^29.
     uint64_t cnt = 0;
@@ -207,9 +213,12 @@ __device__ inline void index_phase(const DPlan& p, const uint8_t* __restrict__ i
     if (threadIdx.x == 0) {
         if (!ok) set_corrupt(p.err);
         if (c == G - 1) {
-            p.tbase[p.nW] = runZ;
+            p.tbase[p.nWi] = runZ;
             *p.n_nctile = (uint32_t)runT;
-            if (runA != hd.nnc || runZ != hd.payload_bytes) set_corrupt(p.err);
+            // totals: exact for the whole stream, bounded for a prefix of it
+            if (p.nWi == p.nW ? (runA != hd.nnc || runZ != hd.payload_bytes)
+                              : (runA > hd.nnc || runZ > hd.payload_bytes))
+                set_corrupt(p.err);
         }
     }
 }
@@ -506,13 +515,22 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
     const uintptr_t lim = reinterpret_cast<uintptr_t>(in) + p.in_bytes;
     const uint64_t nW_full = p.n / ((uint64_t)TB * B);
     const uint32_t slot0 = smem_u32(dsm + (threadIdx.x >> 5) * 2 * C::SLOT_ALLOC);
+    // blocks of tile t inside the requested range [kb0, kb1)
+    auto rmask = [&](uint64_t t) -> uint32_t {
+        uint32_t m = 0xFFFFFFFFu;
+        const uint64_t k0 = t * TB;
+        if (k0 < p.kb0) m &= 0xFFFFFFFFu << (uint32_t)(p.kb0 - k0);
+        if (k0 + TB > p.kb1) m &= (1u << (uint32_t)(p.kb1 - k0)) - 1u;
+        return m;
+    };
+    const uint64_t fill_end = umin64(nW_full, p.nWi);
 
     // ---- fill warps: the constant blocks of every full tile (Fig. 10 state 0:
     // retrieve with mu).  They need only the bitmap word and the tile's mu
     // values, prefetched one tile ahead, so they stream stores.
     auto fill_loop = [&]() {
 #if SZX_FSTATIC
-        uint64_t fnext = ((uint64_t)blockIdx.x * C::FILLW + (threadIdx.x >> 5));
+        uint64_t fnext = p.t_lo + ((uint64_t)blockIdx.x * C::FILLW + (threadIdx.x >> 5));
         auto grab_f = [&]() -> uint64_t {
             const uint64_t v = fnext;
             fnext += (uint64_t)gridDim.x * C::FILLW;
@@ -522,21 +540,21 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
         auto grab_f = [&]() -> uint64_t {
             uint32_t v = 0;
             if (lane == 0) v = atomicAdd(&p.ctr[1], 1u);
-            return __shfl_sync(0xffffffffu, v, 0);
+            return p.t_lo + __shfl_sync(0xffffffffu, v, 0);
         };
 #endif
         uint64_t t = grab_f();
         uint32_t word = 0;
         U mul = 0;
-        if (t < nW_full) { word = bm[t]; mul = mus[t * TB + lane]; }
-        while (t < nW_full) {
+        if (t < fill_end) { word = bm[t]; mul = mus[t * TB + lane]; }
+        while (t < fill_end) {
             const uint64_t tn = grab_f();
             uint32_t wn = 0;
             U mn = 0;
-            if (tn < nW_full) { wn = bm[tn]; mn = mus[tn * TB + lane]; }
+            if (tn < fill_end) { wn = bm[tn]; mn = mus[tn * TB + lane]; }
             uint4* yq = reinterpret_cast<uint4*>(y + t * TB * B + lane * VPL);
 #pragma unroll 2
-            for (uint32_t m = ~word; m; m &= m - 1) {
+            for (uint32_t m = ~word & rmask(t); m; m &= m - 1) {
                 const int j = __ffs(m) - 1;
                 const U mb = __shfl_sync(0xffffffffu, mul, j);
                 T v[VPL];
@@ -639,7 +657,7 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
             if (full) {
                 uint4* yq = reinterpret_cast<uint4*>(y + k0 * B + lane * VPL);
 #pragma unroll 1
-                for (uint32_t m = (SZX_EXP & 2) ? 0u : word; m; m &= m - 1) {
+                for (uint32_t m = (SZX_EXP & 2) ? 0u : (word & rmask(t)); m; m &= m - 1) {
                     const int j = __ffs(m) - 1;
                     const uint32_t r = __popc(word & ((1u << j) - 1u));
                     const uint32_t off = __shfl_sync(0xffffffffu, zoff, r);
@@ -658,9 +676,11 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
                 }
             } else {
                 // last (partial) tile: generic decoder, straight from global memory
+                const uint32_t rm = rmask(t);
                 for (int j = 0; j < TB; j++) {
                     const uint64_t k = k0 + j;
                     if (k >= p.nB) break;
+                    if (!((rm >> j) & 1u)) continue;
                     const int len = (int)umin64(B, p.n - k * B);
                     const T mu = TR::from(__shfl_sync(0xffffffffu, cur.mul, j));
                     T v[VPL];

@@ -184,3 +184,16 @@ def gather_streams(stream: torch.Tensor, records: torch.Tensor, dst: int = 0, gr
 def gather_container(sc: ShardedCompressor, dst: int = 0, group=None) -> torch.Tensor | None:
     """Collect every rank's stream on rank dst and build the SZXC container there."""
     return gather_streams(sc.stream(), sc.records.view(-1, 2), dst, group)
+
+
+def decompress_local(stream: torch.Tensor, n: int, block_size: int, group=None) -> tuple[int, torch.Tensor]:
+    """1 stream -> Q GPUs: this rank reconstructs the block range it would own as
+    shard `rank` of `world` (shard_blocks), from a stream or container held on its device.
+    No collective: each rank reads the bitmap/zsize prefix it needs and decodes its tiles.
+    Returns (first element, values)."""
+    from . import szx as _szx
+    world = dist.get_world_size(group) if dist.is_available() and dist.is_initialized() else 1
+    rank = dist.get_rank(group) if world > 1 else 0
+    nB = (n + block_size - 1) // block_size
+    b0, b1 = shard_blocks(nB, world, rank)
+    return b0 * block_size, _szx.decompress_blocks(stream, b0, b1 - b0)

@@ -57,6 +57,7 @@ def lib() -> ctypes.CDLL:
         "szx_compress_async": (i32, [vp, i32, u64, i32, dbl, u32, vp, u64, vp, u64, vp, vp]),
         "szx_read_header": (i32, [vp, u64, ctypes.POINTER(_Header)]),
         "szx_decompress": (i64, [vp, u64, vp, u64, vp]),
+        "szx_decompress_blocks": (i64, [vp, u64, u64, u64, vp, u64, vp]),
         "szx_decompress_ws": (i64, [vp, u64, vp, u64, vp, u64, vp]),
         "szx_decompress_async": (i32, [vp, u64, ctypes.POINTER(_Header), vp, u64, vp, u64, vp, vp]),
         "szx_compress_host": (i64, [vp, i32, u64, i32, dbl, u32, vp, u64, vp]),
@@ -81,7 +82,7 @@ def lib() -> ctypes.CDLL:
 
 EXPORTED = ["szx_compress_bound", "szx_compress_workspace_bytes", "szx_decompress_workspace_bytes",
             "szx_compress", "szx_compress_ws", "szx_compress_async", "szx_read_header",
-            "szx_decompress", "szx_decompress_ws", "szx_decompress_async", "szx_compress_host",
+            "szx_decompress", "szx_decompress_blocks", "szx_decompress_ws", "szx_decompress_async", "szx_compress_host",
             "szx_decompress_host", "szx_local_range", "szx_compress_shard_async",
             "szx_timing_enable", "szx_timing_reset", "szx_timing_read", "szx_launch_count",
             "szx_debug_set_r_bias", "szx_strerror"]
@@ -185,6 +186,14 @@ def _container_info(stream_t: torch.Tensor):
     return h.n, h.dtype
 
 
+def _block_size(stream_t: torch.Tensor) -> int:
+    head = stream_t[:4].cpu().numpy().tobytes()
+    off = 0
+    if head == b"SZXC":
+        off = struct.unpack_from("<Q", stream_t[48:56].cpu().numpy().tobytes())[0]
+    return struct.unpack_from("<I", stream_t[off + 8:off + 12].cpu().numpy().tobytes())[0]
+
+
 def decompress(s: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
     """Decompress an SZX1 stream or SZXC container held in a uint8 CUDA tensor."""
     _require_cuda(s)
@@ -196,6 +205,26 @@ def decompress(s: torch.Tensor, out: torch.Tensor | None = None, stream=None) ->
                              _stream(stream))
     _check(r, "szx_decompress")
     return out[:n]
+
+
+def decompress_blocks(s: torch.Tensor, first_block: int, n_blocks: int, out: torch.Tensor | None = None,
+                      stream=None) -> torch.Tensor:
+    """Decompress blocks [first_block, first_block + n_blocks) of an SZX1 stream or SZXC container
+    (global block numbering); returns values [first_block*b, min(n, (first_block+n_blocks)*b))."""
+    _require_cuda(s)
+    n, dt = _container_info(s)
+    b = _block_size(s)
+    tdt = torch.float32 if dt == F32 else torch.float64
+    nB = (n + b - 1) // b
+    e0 = min(first_block, nB) * b
+    e1 = min(n, min(nB, first_block + n_blocks) * b)
+    cnt = max(0, e1 - e0)
+    if out is None:
+        out = torch.empty(max(cnt, 1), dtype=tdt, device=s.device)
+    r = lib().szx_decompress_blocks(s.data_ptr(), s.numel(), first_block, n_blocks, out.data_ptr(),
+                                    out.numel() * out.element_size(), _stream(stream))
+    _check(r, "szx_decompress_blocks")
+    return out[:r]
 
 
 def compress_host(x, eb: float, mode="rel", block_size: int = 128, out=None, stream=None):

@@ -89,3 +89,81 @@ def test_sharded_compressor_single_rank_matches_plain_stream():
     c = sdist.gather_container(sc)
     ref = oracle.container_compress(x.cpu().numpy(), 1e-3, oracle.REL, 128, 1)
     assert c.cpu().numpy().tobytes() == ref.tobytes()
+
+
+def _blocks_ref(yref: np.ndarray, b: int, k0: int, nb: int) -> np.ndarray:
+    n = yref.size
+    nB = (n + b - 1) // b
+    e0 = min(k0, nB) * b
+    e1 = min(n, min(nB, k0 + nb) * b)
+    return yref[e0:max(e0, e1)]
+
+
+@pytest.mark.parametrize("dt", [np.float32, np.float64])
+@pytest.mark.parametrize("b", [128, 256])
+def test_decompress_blocks_matches_oracle_slices(dt, b):
+    """1 stream -> Q GPUs: any block range of a stream decodes to the same slice of the oracle's
+    reconstruction, bit for bit (ranges inside one tile, across tiles, unaligned, the tail, empty,
+    clipped at the end)."""
+    x = synth.random_mix(300_007, 7).numpy().astype(dt)  # ragged tail block
+    ref = oracle.compress(x, 1e-3, oracle.REL, b)
+    yref = oracle.decompress(ref)
+    s = torch.from_numpy(ref).cuda()
+    nB = (x.size + b - 1) // b
+    ui = np.uint32 if dt == np.float32 else np.uint64
+    ranges = [(0, nB), (0, 1), (5, 3), (31, 2), (32, 32), (33, 100), (nB - 1, 1), (nB - 40, 1000),
+              (100, 0), (nB, 5), (nB + 3, 1), (7, nB)]
+    for k0, nb in ranges:
+        got = szx.decompress_blocks(s, k0, nb).cpu().numpy()
+        exp = _blocks_ref(yref, b, k0, nb)
+        assert got.size == exp.size, (k0, nb)
+        assert np.array_equal(got.view(ui), exp.view(ui)), (k0, nb)
+
+
+@pytest.mark.parametrize("Q", [2, 3, 8])
+def test_one_stream_to_q_ranks(Q):
+    """A stream written on 1 GPU, decoded by Q ranks (emulated): each rank's block range
+    (shard_blocks) concatenates to the full reconstruction."""
+    x = synth.nyx_like(0, n=96).reshape(-1).contiguous()
+    ref = oracle.compress(x.numpy(), 1e-3, oracle.REL, 128)
+    yref = oracle.decompress(ref)
+    s = torch.from_numpy(ref).cuda()
+    nB = (x.numel() + 127) // 128
+    parts = []
+    for q in range(Q):
+        b0, b1 = sdist.shard_blocks(nB, Q, q)
+        parts.append(szx.decompress_blocks(s, b0, b1 - b0).cpu().numpy())
+    assert np.array_equal(np.concatenate(parts).view(np.uint32), yref.view(np.uint32))
+
+
+@pytest.mark.parametrize("P,Q", [(8, 1), (8, 3), (3, 8), (2, 2)])
+def test_container_block_ranges(P, Q):
+    """A P-shard container decoded as Q block ranges with global block numbering
+    (ranges straddle shard boundaries)."""
+    x = synth.random_mix(200_003, 11).numpy()
+    ref = oracle.container_compress(x, 1e-3, oracle.REL, 128, P)
+    yref = oracle.decompress(ref)
+    c = torch.from_numpy(ref).cuda()
+    nB = (x.size + 127) // 128
+    parts = []
+    for q in range(Q):
+        b0, b1 = sdist.shard_blocks(nB, Q, q)
+        parts.append(szx.decompress_blocks(c, b0, b1 - b0).cpu().numpy())
+    assert np.array_equal(np.concatenate(parts).view(np.uint32), yref.view(np.uint32))
+    got = szx.decompress_blocks(c, 17, 777).cpu().numpy()
+    assert np.array_equal(got.view(np.uint32), _blocks_ref(yref, 128, 17, 777).view(np.uint32))
+
+
+def test_decompress_blocks_errors():
+    x = synth.random_mix(10_000, 5).numpy()
+    ref = oracle.compress(x, 1e-3, oracle.REL, 128)
+    s = torch.from_numpy(ref).cuda()
+    small = torch.empty(10, dtype=torch.float32, device="cuda")
+    with pytest.raises(S.SZxError) as e:
+        szx.decompress_blocks(s, 0, 5, out=small)
+    assert e.value.code == -2  # ENOSPC
+    bad = s.clone()
+    bad[0] = 0
+    with pytest.raises(S.SZxError) as e:
+        szx.decompress_blocks(bad, 0, 5)
+    assert e.value.code == -3  # ECORRUPT
