@@ -234,10 +234,12 @@ def main():
         s0 = codec.out[: codec.stream_bytes()]
     hdr = szx.read_header(s0[:64].cpu().numpy().tobytes())
     S = s0.numel()
-    ref_y = szx.decompress(s0)
-    err = (ref_y.double() - x.double()).abs().max().item()
-    if "SZX_LIB" not in os.environ:  # experiment builds (scripts/run_variants.sh) may skip work
+    if "SZX_LIB" not in os.environ:
+        ref_y = szx.decompress(s0)
+        err = (ref_y.double() - x.double()).abs().max().item()
         assert err <= hdr.eb_abs, (err, hdr.eb_abs)
+    else:  # experiment builds (scripts/run_variants.sh) may skip work or write garbage
+        err = float("nan")
 
     sampler = ClockSampler(local) if rank == 0 else None
     if sampler:

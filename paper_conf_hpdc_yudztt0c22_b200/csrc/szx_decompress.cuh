@@ -373,9 +373,73 @@ __device__ inline bool decode_block_g(const Src src, uint32_t z, int len, T mu,
 // over 32 blocks per warp.
 
 
+// Fast path for the headline shape (float32, b = 128: 4 values per lane),
+// written branch-free: per value one bit-field extract, min/sub for the
+// mid-byte count, a funnel-shift window into the lane's run (two 2-word run
+// loads cover the lane's <= 16 bytes), one LOP3 per map composition, and an
+// unpredicated warp scan of the lead-byte maps (a lane's own map composed
+// with itself is itself, so lanes below the shuffle distance need no guard).
+template <typename Src>
+__device__ __forceinline__ bool decode_full_f32x4(const Src src, uint32_t z, float mu, float (&out)[4]) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t R = src.u8(0);
+    if (R < 9u || R > 32u) return false;
+    const bool raw = R >= 32u;
+    const uint32_t s = raw ? 0u : ((8u - (R & 7u)) & 7u);
+    const uint32_t req = (R + s) >> 3;           // 2..4 kept bytes
+    const uint32_t leads = src.u8(1 + lane);
+    uint32_t m[4], nm[4];
+#pragma unroll
+    for (int i = 0; i < 4; i++) {
+        const uint32_t L = (leads >> (2 * i)) & 3u;
+        const uint32_t copy = L < req ? L : req;
+        m[i] = req - copy;
+        nm[i] = 0xFFFFFFFFu >> (8 * copy);      // bytes NOT copied from the previous value
+    }
+    const uint32_t m01 = m[0] + m[1];
+    const uint32_t msum = m01 + m[2] + m[3];
+    const uint32_t incl = warp_incl_scan(msum);
+    if (33u + __shfl_sync(0xffffffffu, incl, 31) != z) return false;
+    const uint32_t o = 33u + incl - msum;
+    uint32_t ra[2], rb[2];
+    src.template run<2>(o, ra);
+    src.template run<2>(o + m01, rb);
+    const uint32_t drop = 8u * (4u - req);
+    auto lowmask = [](uint32_t mm) { return ~__funnelshift_lc(0u, 0xFFFFFFFFu, 8u * mm); };
+    uint32_t own[4];
+    own[0] = (ra[0] & lowmask(m[0])) << drop;
+    own[1] = (__funnelshift_rc(ra[0], ra[1], 8u * m[0]) & lowmask(m[1])) << drop;
+    own[2] = (rb[0] & lowmask(m[2])) << drop;
+    own[3] = (__funnelshift_rc(rb[0], rb[1], 8u * m[2]) & lowmask(m[3])) << drop;
+    // lane map c -> (c & M) | D
+    uint32_t cM = ~(nm[0] | nm[1] | nm[2] | nm[3]);
+    uint32_t cD = own[0];
+#pragma unroll
+    for (int i = 1; i < 4; i++) cD = (cD & ~nm[i]) | own[i];
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t pM = __shfl_up_sync(0xffffffffu, cM, d);
+        const uint32_t pD = __shfl_up_sync(0xffffffffu, cD, d);
+        cD = (pD & cM) | cD;
+        cM = pM & cM;
+    }
+    uint32_t prev = __shfl_up_sync(0xffffffffu, cD, 1);
+    prev = lane == 0 ? 0u : prev;
+#pragma unroll
+    for (int i = 0; i < 4; i++) {
+        const uint32_t w = (prev & ~nm[i]) | own[i];
+        prev = w;
+        out[i] = raw ? __uint_as_float(w) : __fadd_rn(__uint_as_float(w << s), mu);
+    }
+    return true;
+}
+
 // decode_full with the payload in global memory
 template <typename T, int VPL, typename Src>
 __device__ inline bool decode_full_g(const Src src, uint32_t z, T mu, T (&out)[VPL]) {
+    if constexpr (sizeof(T) == 4 && VPL == 4) {
+        return decode_full_f32x4<Src>(src, z, mu, out);
+    }
     using TR = Traits<T>;
     using U = typename TR::U;
     constexpr int W = TR::W;
@@ -584,26 +648,56 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
         const uint32_t cnt = __popc(m.word);
         m.zl = ((uint32_t)lane < cnt && m.ncb + cnt <= hd.nnc) ? zs[m.ncb + lane] : 0u;
     };
-    // Issue the cp.async copy of (the first SLOT bytes of) a tile's payload
-    // into slot `sl`; returns how many payload bytes, counted from the tile's
-    // first payload byte, the slot holds.
-    auto stage = [&](const TileMeta<U>& m, int sl) -> uint32_t {
-        if (!(m.end > m.base && m.end <= hd.payload_bytes) || (SZX_EXP & 8)) return 0;
-        const uintptr_t g0 = reinterpret_cast<uintptr_t>(pl + m.base);
+    // A tile's payload is decoded in segments of consecutive nonconstant blocks
+    // whose bytes fit one staging slot (a block is at most MAXZ < SLOT bytes):
+    // segment i+1 (of this tile or the next one) is staged with cp.async while
+    // segment i is decoded, so dense tiles never read payload bytes from
+    // global memory inside the decoder.
+    struct SegT {
+        uint32_t r0, r1;   // ranks [r0, r1) among the tile's nonconstant blocks
+        uint32_t off0;     // payload offset of rank r0 within the tile
+    };
+    // per-lane tile facts after validation
+    struct TileZ {
+        uint32_t zl, zincl, cnt;
+        bool ok;
+    };
+    auto tile_z = [&](const TileMeta<U>& m) -> TileZ {
+        TileZ r;
+        r.cnt = __popc(m.word);
+        r.zl = m.zl;
+        bool ok = m.end >= m.base && m.end <= hd.payload_bytes && m.ncb + r.cnt <= hd.nnc;
+        const bool zok = (uint32_t)lane >= r.cnt || (r.zl >= 2 && r.zl <= (uint32_t)MAXZ);
+        r.zincl = warp_incl_scan(r.zl);
+        r.ok = ok && __all_sync(0xffffffffu, zok) && __shfl_sync(0xffffffffu, r.zincl, 31) == m.end - m.base;
+        return r;
+    };
+    // the segment starting at rank r0: as many blocks as fit SLOT - 16 bytes
+    auto seg_from = [&](const TileZ& z, uint32_t r0) -> SegT {
+        SegT sg;
+        sg.r0 = r0;
+        sg.off0 = r0 ? __shfl_sync(0xffffffffu, z.zincl, r0 - 1) : 0u;
+        const bool fits = (uint32_t)lane >= r0 && (uint32_t)lane < z.cnt && z.zincl - sg.off0 <= (uint32_t)(C::SLOT - 16);
+        sg.r1 = r0 + __popc(__ballot_sync(0xffffffffu, fits));
+        if (sg.r1 == r0 && r0 < z.cnt) sg.r1 = r0 + 1;  // (corrupt sizes: validated separately)
+        return sg;
+    };
+    // cp.async the segment's bytes into slot `sl`
+    auto stage_seg = [&](const TileMeta<U>& m, const TileZ& z, const SegT& sg, int sl) {
+        if (!z.ok || (SZX_EXP & 8)) return;
+        const uint32_t off1 = __shfl_sync(0xffffffffu, z.zincl, sg.r1 - 1);
+        const uintptr_t g0 = reinterpret_cast<uintptr_t>(pl + m.base + sg.off0);
         const uintptr_t gA = g0 & ~uintptr_t(15);
-        uintptr_t gE = (reinterpret_cast<uintptr_t>(pl + m.end) + 15) & ~uintptr_t(15);
+        uintptr_t gE = (reinterpret_cast<uintptr_t>(pl + m.base + off1) + 15) & ~uintptr_t(15);
         if (gE > gA + C::SLOT) gE = gA + C::SLOT;
         const uint32_t sa = slot0 + sl * C::SLOT_ALLOC;
         for (uintptr_t a = gA + 16 * lane; a < gE; a += 16 * 32) {
             const uintptr_t rem = lim - a;
             cp_async16_zfill(sa + (uint32_t)(a - gA), reinterpret_cast<const void*>(a), rem < 16 ? (uint32_t)rem : 16u);
         }
-        return (uint32_t)(gE - g0);
     };
-    // dynamic tile assignment: nonconstant-heavy tiles cost far more than
-    // constant ones, so static striding leaves warps idle at the end
-    // nonconstant warps: dynamic assignment over the list of tiles holding
-    // nonconstant blocks (their cost varies far more than the fill's)
+    // dynamic assignment over the list of tiles holding nonconstant blocks
+    // (their cost varies far more than the fill's)
     auto grab = [&]() -> uint64_t {
         uint32_t v = 0xFFFFFFFFu;
         if (lane == 0) {
@@ -613,100 +707,116 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
         v = __shfl_sync(0xffffffffu, v, 0);
         return v == 0xFFFFFFFFu ? p.nW : (uint64_t)v;
     };
+    // decode the blocks of ranks [r0, r1) of a full tile from the staged slot
+    auto decode_seg = [&](uint64_t t, const TileMeta<U>& m, const TileZ& z, const SegT& sg, int sl) {
+        const uint32_t sbase = slot0 + sl * C::SLOT_ALLOC +
+                               (uint32_t)(reinterpret_cast<uintptr_t>(pl + m.base + sg.off0) & 15) - sg.off0;
+        uint4* yq = reinterpret_cast<uint4*>(y + t * TB * B + lane * VPL);
+        const uint32_t rm = rmask(t);
+        // blocks whose rank lies in [r0, r1): clear the set bits below r0 and from r1 on
+        uint32_t sel = m.word;
+        for (uint32_t r = 0; r < sg.r0; r++) sel &= sel - 1;
+        uint32_t keep = sel;
+        for (uint32_t r = sg.r0; r < sg.r1; r++) keep &= keep - 1;
+        sel &= ~keep;
+        uint32_t r = sg.r0;
+#pragma unroll 1
+        for (uint32_t bits = (SZX_EXP & 2) ? 0u : sel; bits; bits &= bits - 1, r++) {
+            const int j = __ffs(bits) - 1;
+            const uint32_t off = __shfl_sync(0xffffffffu, z.zincl - z.zl, r);
+            const uint32_t zz = __shfl_sync(0xffffffffu, z.zl, r);
+            const T mu = TR::from(__shfl_sync(0xffffffffu, m.mul, j));
+            if (!((rm >> j) & 1u)) continue;
+            T v[VPL];
+            if (!decode_full_g<T, VPL>(SrcS{sbase + off}, zz, mu, v)) {
+                if (lane == 0) set_corrupt(p.err);
+                continue;
+            }
+#pragma unroll
+            for (int q = 0; q < NV; q++) st_out16(yq + j * QB + q, reinterpret_cast<const uint4*>(v)[q]);
+        }
+    };
+    // the partial last tile: generic decoder, straight from global memory
+    auto decode_partial = [&](uint64_t t, const TileMeta<U>& m, const TileZ& z) {
+        const uint64_t k0 = t * TB;
+        const uint32_t rm = rmask(t);
+        const uint8_t* gb = pl + m.base;
+        for (int j = 0; j < TB; j++) {
+            const uint64_t k = k0 + j;
+            if (k >= p.nB) break;
+            if (!((rm >> j) & 1u)) continue;
+            const int len = (int)umin64(B, p.n - k * B);
+            const T mu = TR::from(__shfl_sync(0xffffffffu, m.mul, j));
+            T v[VPL];
+            if (!((m.word >> j) & 1u)) {
+#pragma unroll
+                for (int q = 0; q < VPL; q++) v[q] = mu;
+            } else {
+                const uint32_t r = __popc(m.word & ((1u << j) - 1u));
+                const uint32_t off = __shfl_sync(0xffffffffu, z.zincl - z.zl, r);
+                const uint32_t zz = __shfl_sync(0xffffffffu, z.zl, r);
+                if (!decode_block_g<T, VPL>(SrcG{gb + off, lim}, zz, len, mu, v)) {
+                    if (lane == 0) set_corrupt(p.err);
+                    continue;
+                }
+            }
+            store_lane<T, VPL>(y, p.n, k, lane, v);
+        }
+    };
 
     auto nc_loop = [&]() {
-    uint64_t t = grab();
-    if (t >= p.nW) return;
-    TileMeta<U> cur, nx;
-    load_meta(t, cur);
-    load_zl(cur);
-    uint32_t cur_staged = stage(cur, 0);
-    cp_async_commit();
-    int sl = 0;
-    while (t < p.nW) {
-        const uint64_t tn = grab();
-        if (tn < p.nW) load_meta(tn, nx);
-        // validate the current tile's metadata
-        const uint32_t word = cur.word;
-        const uint32_t cnt = __popc(word);
-        bool ok = cur.end >= cur.base && cur.end <= hd.payload_bytes && cur.ncb + cnt <= hd.nnc;
-        const uint32_t zl = cur.zl;
-        const bool zok = (uint32_t)lane >= cnt || (zl >= 2 && zl <= (uint32_t)MAXZ);
-        const uint32_t zincl = warp_incl_scan(zl);
-        ok = ok && __all_sync(0xffffffffu, zok) && __shfl_sync(0xffffffffu, zincl, 31) == cur.end - cur.base;
-        const uint32_t zoff = zincl - zl;
-        const uint64_t k0 = t * TB;
-        const bool full = t < nW_full;
-        // prefetch the next tile's payload into the other slot
-        uint32_t nx_staged = 0;
-        if (tn < p.nW) {
-            load_zl(nx);
-            nx_staged = stage(nx, sl ^ 1);
-        }
+        uint64_t t = grab();
+        if (t >= p.nW) return;
+        TileMeta<U> cur, nx;
+        load_meta(t, cur);
+        load_zl(cur);
+        TileZ cz = tile_z(cur);
+        SegT sg = seg_from(cz, 0);
+        const bool cfull0 = t < nW_full;
+        if (cfull0 && cz.ok && cz.cnt) stage_seg(cur, cz, sg, 0);
         cp_async_commit();
-        cp_async_wait<1>();
-        __syncwarp();
-        if (!ok) {
-            if (lane == 0) set_corrupt(p.err);
-        } else {
-            // nonconstant payloads: from the staging slot when the block lies
-            // inside the staged prefix, else straight from global memory
-            const uint32_t sbase = slot0 + sl * C::SLOT_ALLOC +
-                                   (uint32_t)(reinterpret_cast<uintptr_t>(pl + cur.base) & 15);
-            const uint8_t* gbase = pl + cur.base;
-            if (full) {
-                uint4* yq = reinterpret_cast<uint4*>(y + k0 * B + lane * VPL);
-#pragma unroll 1
-                for (uint32_t m = (SZX_EXP & 2) ? 0u : (word & rmask(t)); m; m &= m - 1) {
-                    const int j = __ffs(m) - 1;
-                    const uint32_t r = __popc(word & ((1u << j) - 1u));
-                    const uint32_t off = __shfl_sync(0xffffffffu, zoff, r);
-                    const uint32_t z = __shfl_sync(0xffffffffu, zl, r);
-                    const T mu = TR::from(__shfl_sync(0xffffffffu, cur.mul, j));
-                    T v[VPL];
-                    bool good;
-                    if (off + z <= cur_staged) good = decode_full_g<T, VPL>(SrcS{sbase + off}, z, mu, v);
-                    else good = decode_full_g<T, VPL>(SrcG{gbase + off, lim}, z, mu, v);
-                    if (!good) {
-                        if (lane == 0) set_corrupt(p.err);
-                        continue;
-                    }
-#pragma unroll
-                    for (int q = 0; q < NV; q++) st_out16(yq + j * QB + q, reinterpret_cast<const uint4*>(v)[q]);
-                }
+        uint64_t tn = grab();
+        if (tn < p.nW) load_meta(tn, nx);
+        int sl = 0;
+        while (t < p.nW) {
+            const bool cfull = t < nW_full;
+            if (!cz.ok && lane == 0) set_corrupt(p.err);
+            // the next work item: the rest of this tile, or the next tile
+            bool next_same = cfull && cz.ok && sg.r1 < cz.cnt;
+            TileZ nz = cz;
+            SegT ns = sg;
+            if (next_same) {
+                ns = seg_from(cz, sg.r1);
+                stage_seg(cur, cz, ns, sl ^ 1);
+            } else if (tn < p.nW) {
+                load_zl(nx);
+                nz = tile_z(nx);
+                ns = seg_from(nz, 0);
+                if (tn < nW_full && nz.ok && nz.cnt) stage_seg(nx, nz, ns, sl ^ 1);
+            }
+            cp_async_commit();
+            cp_async_wait<1>();
+            __syncwarp();
+            if (cz.ok) {
+                if (cfull) decode_seg(t, cur, cz, sg, sl);
+                else decode_partial(t, cur, cz);
+            }
+            __syncwarp();  // slot `sl` is refilled by the item after next
+            sl ^= 1;
+            if (next_same) {
+                sg = ns;
             } else {
-                // last (partial) tile: generic decoder, straight from global memory
-                const uint32_t rm = rmask(t);
-                for (int j = 0; j < TB; j++) {
-                    const uint64_t k = k0 + j;
-                    if (k >= p.nB) break;
-                    if (!((rm >> j) & 1u)) continue;
-                    const int len = (int)umin64(B, p.n - k * B);
-                    const T mu = TR::from(__shfl_sync(0xffffffffu, cur.mul, j));
-                    T v[VPL];
-                    if (!((word >> j) & 1u)) {
-#pragma unroll
-                        for (int q = 0; q < VPL; q++) v[q] = mu;
-                    } else {
-                        const uint32_t r = __popc(word & ((1u << j) - 1u));
-                        const uint32_t off = __shfl_sync(0xffffffffu, zoff, r);
-                        const uint32_t z = __shfl_sync(0xffffffffu, zl, r);
-                        if (!decode_block_g<T, VPL>(SrcG{gbase + off, lim}, z, len, mu, v)) {
-                            if (lane == 0) set_corrupt(p.err);
-                            continue;
-                        }
-                    }
-                    store_lane<T, VPL>(y, p.n, k, lane, v);
+                t = tn;
+                cur = nx;
+                cz = nz;
+                sg = ns;
+                if (t < p.nW) {
+                    tn = grab();
+                    if (tn < p.nW) load_meta(tn, nx);
                 }
             }
         }
-        __syncwarp();  // slot `sl` is refilled two tiles from now
-        cur = nx;
-        cur_staged = nx_staged;
-        sl ^= 1;
-        t = tn;
-    }
-    cp_async_wait<0>();
+        cp_async_wait<0>();
     };
     // Each warp drains its own queue first, then helps with the other one, so
     // the split adapts to the field's fraction of nonconstant blocks.
