@@ -152,9 +152,7 @@ CLayout clayout(uint64_t n, int W, uint32_t b) {
     L.nB = cdiv(n, b);
     L.nW = cdiv(L.nB, 32);
     L.nTB = cdiv(L.nB, kClassifyBlocks);
-    // look-back status words: k_zscan CTAs (split encoder) or fused-encoder tiles
-    // (32 * 512 / (b W) blocks each), whichever is more
-    L.nTC = std::max<uint64_t>(cdiv(cdiv(L.nB, kWriteTile), 256), cdiv(L.nB, 32ull * 512 / ((uint64_t)b * W)));
+    L.nTC = cdiv(cdiv(L.nB, kWriteTile), 256);  // k_zscan CTAs (look-back status words)
     L.off_keys = 0;
     L.off_zero = 16;
     L.zero_bytes = al16(16 + 8 * L.nTB + 8 * L.nTC);
@@ -225,8 +223,6 @@ void set_smem_attrs() {
     carve(k_decode_w<T, VPL>);
     cudaFuncSetAttribute(k_enc_write<T, VPL>, cudaFuncAttributeMaxDynamicSharedMemorySize, WriteCfg<T, VPL>::SMEM);
     cudaFuncSetAttribute(k_enc_size<T, VPL>, cudaFuncAttributeMaxDynamicSharedMemorySize, SizeCfg<T, VPL>::SMEM);
-    cudaFuncSetAttribute(k_encode<T, VPL>, cudaFuncAttributeMaxDynamicSharedMemorySize, EncCfg<T, VPL>::SMEM);
-    carve(k_encode<T, VPL>);
 
     done = true;
 }
@@ -258,22 +254,6 @@ template <typename T, int VPL>
 void enqueue_encode(const void* d_in, const Plan& p, const CLayout& L, uint8_t* out, cudaStream_t s) {
     set_smem_attrs<T, VPL>();
     launch("k_classify", s, [&] { launch_pdl(k_classify<T>, dim3((unsigned)L.nTB), dim3(256), 0, s, p, out); });
-#ifndef SZX_SPLIT_ENC
-    {   // fused single-pass encoder: persistent CTAs, at most one per tile
-        using E = EncCfg<T, VPL>;
-        static int eocc = 0;
-        if (!eocc) {
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&eocc, k_encode<T, VPL>, 256, E::SMEM);
-            if (eocc <= 0) eocc = 1;
-        }
-        uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * eocc, cdiv(L.nB, E::TB));
-        if (grid == 0) grid = 1;
-        launch("k_encode", s, [&] {
-            launch_pdl(k_encode<T, VPL>, dim3((unsigned)grid), dim3(256), E::SMEM, s, static_cast<const T*>(d_in), p, out);
-        });
-        return;
-    }
-#endif
     static int occ = 0;
     if (!occ) {
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_enc_size<T, VPL>, 256, SizeCfg<T, VPL>::SMEM);

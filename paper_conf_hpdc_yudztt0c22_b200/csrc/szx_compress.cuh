@@ -464,7 +464,11 @@ __device__ inline uint32_t size_block(const T (&xv)[VPL], T mu, int& R, bool pro
 // without byte stores or run assembly.  dst is the shared-memory address of
 // the block payload; values [0, cnt) of the lane are valid, len in the block.
 __device__ inline void red_or_s(uint32_t a, uint32_t v) {
+#ifdef SZX_EXP_STS
+    asm volatile("st.shared.b32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+#else
     asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+#endif
 }
 __device__ inline void red_or_byte(uint32_t a, uint32_t v) { red_or_s(a & ~3u, (v & 0xFFu) << (8 * (a & 3u))); }
 
@@ -508,6 +512,125 @@ __device__ inline void pack_red(const typename Traits<T>::U (&u)[VPL], const Lan
             }
             a += mi;
         }
+    }
+}
+
+// R2 guard / escalation only (R2): returns the final R of a block
+// whose per-element check was not proven unnecessary by classify.
+template <typename T, int VPL>
+__device__ inline int guard_R(const T (&xv)[VPL], int cnt, T mu, int R, double eb) {
+    using TR = Traits<T>;
+    using U = typename TR::U;
+    constexpr int W = TR::W;
+    for (;;) {
+        if (R >= TR::kFull) return TR::kFull;
+        const int s = (8 - (R & 7)) & 7;
+        const U keep = ~((U(1) << (8 * W - R)) - U(1));
+        bool ok = true;
+#pragma unroll
+        for (int i = 0; i < VPL; i++) {
+            if (i < cnt) {
+                const U u = TR::bits(TR::sub(xv[i], mu)) >> s;
+                const T xp = TR::add(TR::from((u << s) & keep), mu);
+                ok &= fabs(__dsub_rn((double)xv[i], (double)xp)) <= eb;
+            }
+        }
+        if (__all_sync(0xffffffffu, ok)) return R;
+        R += 1;
+    }
+}
+
+// ---------------------------------------------------------- float32 fast path
+// Full float32 blocks of b = 128 (4 values per lane) with a FINAL R (the guard
+// has run): shifted words, lead codes and the per-value mid-byte counts, all
+// branch-free.  Identical output to encode_block/encode_known_R.
+struct Lane4 {
+    uint32_t u[4];      // shifted words
+    uint32_t leads;     // 2-bit codes, LSB-first
+    uint32_t msum;      // mid-bytes of this lane (consumed by the scan)
+};
+__device__ __forceinline__ void lane_encode_f32x4(const float (&xv)[4], float mu, int R, Lane4& e) {
+    const int lane = threadIdx.x & 31;
+    const bool raw = R >= 32;
+    const uint32_t s = raw ? 0u : ((8u - ((uint32_t)R & 7u)) & 7u);
+    const uint32_t req = ((uint32_t)R + s) >> 3;
+#pragma unroll
+    for (int i = 0; i < 4; i++)
+        e.u[i] = (raw ? __float_as_uint(xv[i]) : __float_as_uint(__fsub_rn(xv[i], mu))) >> s;
+    uint32_t prev = __shfl_up_sync(0xffffffffu, e.u[3], 1);
+    prev = lane == 0 ? 0u : prev;
+    uint32_t leads = 0, msum = 0;
+#pragma unroll
+    for (int i = 0; i < 4; i++) {
+        const uint32_t L = umin_(3u, (uint32_t)__clz(e.u[i] ^ prev) >> 3);
+        prev = e.u[i];
+        leads |= L << (2 * i);
+        msum += req - umin_(L, req);
+    }
+    e.leads = leads;
+    e.msum = msum;
+}
+
+// Mid-bytes of this lane only (the size pass): no codes kept.
+__device__ __forceinline__ uint32_t lane_msum_f32x4(const float (&xv)[4], float mu, int R) {
+    const int lane = threadIdx.x & 31;
+    const bool raw = R >= 32;
+    const uint32_t s = raw ? 0u : ((8u - ((uint32_t)R & 7u)) & 7u);
+    const uint32_t req = ((uint32_t)R + s) >> 3;
+    uint32_t u[4];
+#pragma unroll
+    for (int i = 0; i < 4; i++) u[i] = (raw ? __float_as_uint(xv[i]) : __float_as_uint(__fsub_rn(xv[i], mu))) >> s;
+    uint32_t prev = __shfl_up_sync(0xffffffffu, u[3], 1);
+    prev = lane == 0 ? 0u : prev;
+    uint32_t msum = 0;
+#pragma unroll
+    for (int i = 0; i < 4; i++) {
+        const uint32_t L = umin_(3u, (uint32_t)__clz(u[i] ^ prev) >> 3);
+        prev = u[i];
+        msum += req - umin_(L, req);
+    }
+    return msum;
+}
+
+// OR v into shared word a unless v == 0 (predicated, no branch)
+__device__ __forceinline__ void red_or_nz(uint32_t a, uint32_t v) {
+#ifdef SZX_EXP_STS
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %1, 0;\n\t@q st.shared.b32 [%0], %1;\n\t}"
+                 ::"r"(a), "r"(v) : "memory");
+#else
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %1, 0;\n\t@q red.shared.or.b32 [%0], %1;\n\t}"
+                 ::"r"(a), "r"(v) : "memory");
+#endif
+}
+// Pack a full float32 block into a zeroed shared staging area at byte address
+// dst: [R][32 code bytes][mid-bytes].  Values are placed in pairs: the two
+// chunks (<= 8 bytes) are joined with funnel shifts and OR-ed in as at most
+// three aligned words.
+__device__ __forceinline__ void lane_pack_f32x4(const Lane4& e, int R, uint32_t mexcl, uint32_t dst) {
+    const int lane = threadIdx.x & 31;
+    if (lane == 0) red_or_s(dst & ~3u, (uint32_t)R << (8 * (dst & 3u)));
+    {
+        const uint32_t a = dst + 1 + lane;
+        red_or_s(a & ~3u, e.leads << (8 * (a & 3u)));
+    }
+    const bool raw = R >= 32;
+    const uint32_t s = raw ? 0u : ((8u - ((uint32_t)R & 7u)) & 7u);
+    const uint32_t req = ((uint32_t)R + s) >> 3;
+    const uint32_t drop = 8u * (4u - req);
+    uint32_t a = dst + 33 + mexcl;
+#pragma unroll
+    for (int h = 0; h < 2; h++) {
+        const uint32_t m0 = req - umin_((e.leads >> (4 * h)) & 3u, req);
+        const uint32_t m1 = req - umin_((e.leads >> (4 * h + 2)) & 3u, req);
+        const uint32_t c0 = (e.u[2 * h] >> drop) & ~__funnelshift_lc(0u, 0xFFFFFFFFu, 8 * m0);
+        const uint32_t c1 = (e.u[2 * h + 1] >> drop) & ~__funnelshift_lc(0u, 0xFFFFFFFFu, 8 * m1);
+        const uint32_t lo = c0 | __funnelshift_lc(0u, c1, 8 * m0);
+        const uint32_t hi = __funnelshift_lc(c1, 0u, 8 * m0);
+        const uint32_t sh = 8 * (a & 3u), wa = a & ~3u;
+        red_or_nz(wa, lo << sh);
+        red_or_nz(wa + 4, __funnelshift_l(lo, hi, sh));
+        red_or_nz(wa + 8, __funnelshift_l(hi, 0u, sh));
+        a += m0 + m1;
     }
 }
 
@@ -606,8 +729,18 @@ __global__ void __launch_bounds__(256) k_enc_size(const T* __restrict__ x, Plan 
                         reinterpret_cast<uint4*>(x1)[q] = lds_u128(st + (j + 1) * C::BW + (lane * C::QV + q) * 16);
                     }
                     int R0 = (int)(rec0 & 0x7F), R1 = (int)(rec1 & 0x7F);
-                    const uint32_t z0 = size_block<T, VPL>(x0, mu0, R0, (rec0 & 0x80) != 0, eb);
-                    const uint32_t z1 = two ? size_block<T, VPL>(x1, mu1, R1, (rec1 & 0x80) != 0, eb) : 0u;
+                    uint32_t z0, z1 = 0u;
+                    if constexpr (sizeof(T) == 4 && VPL == 4) {
+                        if (!(rec0 & 0x80)) R0 = guard_R<T, VPL>(x0, VPL, mu0, R0, eb);
+                        if (two && !(rec1 & 0x80)) R1 = guard_R<T, VPL>(x1, VPL, mu1, R1, eb);
+                        const uint32_t m0 = lane_msum_f32x4(x0, mu0, R0);
+                        const uint32_t m1 = lane_msum_f32x4(x1, mu1, R1);
+                        z0 = 33u + warp_sum(m0);
+                        if (two) z1 = 33u + warp_sum(m1);
+                    } else {
+                        z0 = size_block<T, VPL>(x0, mu0, R0, (rec0 & 0x80) != 0, eb);
+                        z1 = two ? size_block<T, VPL>(x1, mu1, R1, (rec1 & 0x80) != 0, eb) : 0u;
+                    }
                     if (lane == 0) {
                         zsize[nc] = (uint16_t)z0;
                         p.ncR[nc] = (uint8_t)R0;
@@ -830,8 +963,15 @@ __global__ void __launch_bounds__(256) k_enc_write(const T* __restrict__ x, Plan
 #pragma unroll
             for (int q = 0; q < C::QV; q++)
                 reinterpret_cast<uint4*>(xv)[q] = lds_u128(sin + j * C::BW + (lane * C::QV + q) * 16);
-            encode_known_R<T, VPL>(xv, VPL, C::B, cmu, R, u, lc);
-            pack_red<T, VPL>(u, lc, VPL, C::B, smem_u32(stg) + sb + zo);
+            if constexpr (sizeof(T) == 4 && VPL == 4) {
+                Lane4 e;
+                lane_encode_f32x4(xv, cmu, R, e);
+                const uint32_t incl = warp_incl_scan(e.msum);
+                lane_pack_f32x4(e, R, incl - e.msum, smem_u32(stg) + sb + zo);
+            } else {
+                encode_known_R<T, VPL>(xv, VPL, C::B, cmu, R, u, lc);
+                pack_red<T, VPL>(u, lc, VPL, C::B, smem_u32(stg) + sb + zo);
+            }
         } else {  // the partial tail block
             const int cnt = load_lane<T, VPL>(x, p.n, k, lane, xv);
             const int len = (int)(p.n - (uint64_t)k * C::B);
@@ -855,278 +995,6 @@ __global__ void __launch_bounds__(256) k_enc_write(const T* __restrict__ x, Plan
             for (int q = 0; q < 16; q++)
                 if (a + q >= a0 && a + q < E) *reinterpret_cast<uint8_t*>(a + q) = vb[q];
         }
-    }
-}
-
-// ------------------------------------------------------------------ K2 fused encoder
-// Single pass over the nonconstant blocks (compacted list): for every tile of
-// TB blocks the CTA encodes (Formula 4 R from classify, R2 guard / escalation,
-// Formula 5 shift, lead codes, mid-byte counts -> z_k), publishes the tile's
-// payload size for a decoupled look-back (Merrill & Garland) before packing,
-// packs [R][codes][mid-bytes] with shared-memory OR reductions into a zeroed
-// staging area, resolves the tile's payload offset and copies the staged bytes
-// out realigned to that offset with 16-byte stores.  This is the paper's
-// "zsize + prefix sum" done in the same pass as the encoding.
-// Persistent CTAs take tiles by atomic ticket (so every predecessor of a tile
-// is resident or done: the look-back always progresses) and prefetch the next
-// tile's values with cp.async while the current one is encoded.
-template <typename T, int VPL>
-struct EncCfg {
-    static constexpr int W = Traits<T>::W;
-    static constexpr int B = 32 * VPL;
-    static constexpr int BW = B * W;
-    static constexpr int QV = VPL * W / 16;          // 16-byte chunks per lane per block
-    static constexpr int NWARP = 8;
-    static constexpr int TB = 32 * 512 / BW;         // blocks per tile: 32 (f32, b=128), 16, 8
-    static constexpr int BPW = TB / NWARP;           // blocks per warp
-    static constexpr int MAXZ = 1 + B / 4 + W * B;
-    static constexpr int STG = (16 + TB * MAXZ + 48 + 15) / 16 * 16;  // zero lead pad + payload + read pad
-    static constexpr int IN = TB * BW;
-    static constexpr int NSTG = 3;                   // staging areas in rotation (pack, copy-out, re-zero)
-    static constexpr int SMEM = NSTG * STG + IN;
-    static_assert(TB <= 32 && BPW >= 1, "tile must fit one warp scan");
-};
-
-// Round-synchronous tile offsets.  With the static schedule, round r holds
-// tiles [rG, rG + G) (one per CTA).  Each tile publishes its payload size
-// (flag bit 63 | bytes) as soon as it is encoded; one iteration later every
-// CTA reads the whole round's sizes (each warp a slice, loads issued before
-// packing and consumed after it, so their latency is hidden), takes the
-// prefix up to its own tile, and advances its running base by the round
-// total.  No tile waits on a chain of predecessors, and the sizes are
-// normally all published by the time they are read (a lagging CTA is waited
-// for).  Requires a co-resident grid.
-__device__ inline void round_publish(uint64_t* slots, uint64_t tile, uint32_t bytes) {
-    st_relaxed(&slots[tile], (1ull << 63) | bytes);
-}
-template <typename T, int VPL>
-__global__ void __launch_bounds__(256, 3) k_encode(const T* __restrict__ x, Plan p, uint8_t* __restrict__ out) {
-    using TR = Traits<T>;
-    using U = typename TR::U;
-    using C = EncCfg<T, VPL>;
-    constexpr int W = TR::W;
-    constexpr int B = C::B;
-    constexpr int TB = C::TB;
-    constexpr int BPW = C::BPW;
-    extern __shared__ __align__(16) uint8_t smem[];
-    __shared__ uint32_t s_z[TB];
-    __shared__ uint64_t s_pre[8], s_tot[8];
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const uint32_t stg0 = smem_u32(smem), in0 = stg0 + C::NSTG * C::STG;
-    // zero the staging areas once; afterwards each is re-zeroed after its copy-out
-    for (uint32_t ch = threadIdx.x; ch < C::NSTG * C::STG / 16; ch += 256)
-        reinterpret_cast<uint4*>(smem)[ch] = make_uint4(0, 0, 0, 0);
-    pdl_wait();
-    pdl_trigger();
-    const uint64_t nnc = *p.nnc;
-    const double eb = *p.eb_abs;
-    const uint64_t ntiles = (nnc + TB - 1) / TB;
-    const uint64_t off_zs = p.off_mu + al16((uint64_t)W * p.nB);
-    const uint64_t off_pl = off_zs + al16(2 * nnc);
-    uint16_t* zsize = reinterpret_cast<uint16_t*>(out + off_zs);
-    U* mus = reinterpret_cast<U*>(out + p.off_mu);
-    const U* ncmu = reinterpret_cast<const U*>(p.ncmu);
-    const uint64_t nBfull = p.n / B;
-    __syncthreads();
-    // static round robin over the co-resident grid: CTA c takes tiles c, c+G, ...
-    uint64_t t = blockIdx.x;
-    if (t >= ntiles) return;
-
-    // metadata of the warp's BPW blocks of tile tt (lane j < BPW holds block j)
-    struct Meta { uint32_t k, rec; U mu; };
-    auto meta = [&](uint64_t tt) -> Meta {
-        const uint64_t nc = tt * TB + warp * BPW + lane;
-        Meta m{0u, 0u, U(0)};
-        if (lane < BPW && nc < nnc) { m.k = p.nclist[nc]; m.mu = ncmu[nc]; m.rec = p.ncR[nc]; }
-        return m;
-    };
-    // cp.async of the warp's blocks of tile tt into the input buffer
-    auto issue = [&](uint64_t tt, const Meta& m) {
-        const uint32_t dst = in0 + warp * BPW * C::BW;
-#pragma unroll
-        for (int j = 0; j < BPW; j++) {
-            const uint32_t k = __shfl_sync(0xffffffffu, m.k, j);
-            if (tt * TB + warp * BPW + j < nnc && k < nBfull) {
-                const T* src = x + (uint64_t)k * B + lane * VPL;
-#pragma unroll
-                for (int q = 0; q < C::QV; q++) cp_async16(dst + j * C::BW + (lane * C::QV + q) * 16, src + q * (16 / W));
-            }
-        }
-        cp_async_commit();
-    };
-    // copy a staged tile (Tb bytes at staging offset 16) to its payload offset,
-    // realigned, with 16-byte stores (byte stores in the two boundary chunks,
-    // which the neighbouring tiles share)
-    auto copy_out = [&](uint32_t sp, uint64_t tt, uint64_t base, uint32_t Tb) {
-        const uint64_t g0 = off_pl + base;
-        const uint32_t mis = (uint32_t)(g0 & 15);
-        const uint64_t A0 = g0 - mis;
-        const uint32_t nch = (mis + Tb + 15) >> 4;
-        for (uint32_t ch = threadIdx.x; ch < nch; ch += 256) {
-            uint32_t r[4];
-            run_load_s<4>(sp + 16 * ch - mis, r);
-            uint8_t* dst = out + A0 + 16 * (uint64_t)ch;
-            const int64_t lo = (int64_t)mis - 16 * (int64_t)ch, hi = (int64_t)mis + Tb - 16 * (int64_t)ch;
-            if (lo <= 0 && hi >= 16) {
-                *reinterpret_cast<uint4*>(dst) = make_uint4(r[0], r[1], r[2], r[3]);
-            } else {
-#pragma unroll
-                for (int q = 0; q < 16; q++)
-                    if (q >= lo && q < hi) dst[q] = (uint8_t)(r[q >> 2] >> (8 * (q & 3)));
-            }
-        }
-        if (tt == ntiles - 1 && threadIdx.x == 0) {
-            const uint64_t pbytes = base + Tb;
-            reinterpret_cast<uint64_t*>(out)[6] = pbytes;  // header: payload bytes
-            *p.total = off_pl + pbytes;
-        }
-    };
-    Meta cur = meta(t), nxt{0u, 0u, U(0)};
-    issue(t, cur);
-    // Software pipeline: tile i is encoded, published and packed in iteration
-    // i, its offset resolved and its bytes copied out in iteration i+1 (by
-    // then its predecessors have published), and its staging area re-zeroed
-    // in iteration i+2.  Three staging areas rotate.
-    uint64_t t_prev = 0;
-    uint64_t run_base = 0;  // payload bytes of all rounds before t_prev's
-    uint32_t tb_prev = 0, tb_pp = 0;
-    int it = 0;
-    for (;; it++) {
-        const int sb = it % C::NSTG;
-        const uint64_t tn = t + gridDim.x;
-        if (tn < ntiles) nxt = meta(tn);  // used after barrier #1
-        cp_async_wait<0>();
-        __syncwarp();
-        // ---- encode the warp's blocks (registers)
-        U u[BPW][VPL];
-        LaneCode lc[BPW];
-#pragma unroll
-        for (int j = 0; j < BPW; j++) {
-            const uint64_t nc = t * TB + warp * BPW + j;
-            lc[j].z = 0;
-            lc[j].R = 0;
-            if (nc < nnc) {
-                const uint32_t k = __shfl_sync(0xffffffffu, cur.k, j);
-                const T mu = TR::from(__shfl_sync(0xffffffffu, cur.mu, j));
-                const uint32_t rec = __shfl_sync(0xffffffffu, cur.rec, j);
-                T xv[VPL];
-                if (k < nBfull) {
-                    const uint32_t sa = in0 + (warp * BPW + j) * C::BW;
-#pragma unroll
-                    for (int q = 0; q < C::QV; q++)
-                        reinterpret_cast<uint4*>(xv)[q] = lds_u128(sa + (lane * C::QV + q) * 16);
-                    encode_block<T, VPL>(xv, VPL, B, mu, (int)(rec & 0x7F), (rec & 0x80) != 0, eb, u[j], lc[j]);
-                } else {  // the partial tail block, straight from global memory
-                    const int cnt = load_lane<T, VPL>(x, p.n, k, lane, xv);
-                    const int len = (int)(p.n - (uint64_t)k * B);
-                    encode_block<T, VPL>(xv, cnt, len, mu, (int)(rec & 0x7F), (rec & 0x80) != 0, eb, u[j], lc[j]);
-                }
-                if (lane == 0 && lc[j].R >= TR::kFull) mus[k] = 0;  // raw: mu = +0 (R15)
-            }
-            if (lane == 0) s_z[warp * BPW + j] = lc[j].z;
-        }
-        __syncthreads();  // #1: s_z complete, the input buffer is free
-        if (tn < ntiles) issue(tn, nxt);
-        // tile scan of z (every warp, redundantly) -> in-tile offsets, tile size
-        const uint32_t zl = lane < TB ? s_z[lane] : 0u;
-        const uint32_t zincl = warp_incl_scan(zl);
-        const uint32_t Tb = __shfl_sync(0xffffffffu, zincl, 31);
-        if (threadIdx.x == 0) round_publish(p.status_c, t, Tb);
-        if (threadIdx.x < TB && t * TB + threadIdx.x < nnc) zsize[t * TB + threadIdx.x] = (uint16_t)zl;
-        {   // re-zero the staging area of the tile copied out last iteration
-            const uint32_t sz = stg0 + ((it + 1) % C::NSTG) * C::STG;
-            const uint32_t nch = (16 + tb_pp + 48 + 15) >> 4;
-            for (uint32_t ch = threadIdx.x; ch < nch; ch += 256)
-                asm volatile("st.shared.v4.u32 [%0], {%1,%1,%1,%1};" ::"r"(sz + 16 * ch), "r"(0u) : "memory");
-        }
-        // ---- the previous tile's round: this warp's slice of the published sizes
-        constexpr int QW = 3;  // entries per lane: G <= 8 warps x 32 x QW
-        const uint64_t G = gridDim.x;
-        const uint64_t per_w = (G + 7) / 8;
-        const uint64_t r0 = t_prev / G * G, r1 = umin64(r0 + G, ntiles);
-        uint64_t rv[QW];
-#pragma unroll
-        for (int q = 0; q < QW; q++) {
-            const uint64_t o = 32 * q + lane, idx = r0 + warp * per_w + o;
-            rv[q] = (it > 0 && o < per_w && idx < r1) ? ld_relaxed(&p.status_c[idx]) : (1ull << 63);
-        }
-        // ---- pack into the zeroed staging area (16-byte lead pad)
-        const uint32_t sp = stg0 + sb * C::STG + 16;
-#pragma unroll
-        for (int j = 0; j < BPW; j++) {
-            const int bi = warp * BPW + j;
-            const uint64_t nc = t * TB + bi;
-            const uint32_t zo = __shfl_sync(0xffffffffu, zincl - zl, bi);
-            if (nc < nnc) {
-                const uint32_t k = __shfl_sync(0xffffffffu, cur.k, j);
-                if (k < nBfull) {
-                    pack_red<T, VPL>(u[j], lc[j], VPL, B, sp + zo);
-                } else {
-                    const uint64_t first = (uint64_t)k * B + (uint64_t)lane * VPL;
-                    const int cnt = first >= p.n ? 0 : (int)umin64(VPL, p.n - first);
-                    pack_red<T, VPL>(u[j], lc[j], cnt, (int)(p.n - (uint64_t)k * B), sp + zo);
-                }
-            }
-        }
-        // ---- the previous tile: offset (sum of the slices), then copy-out
-        {
-            uint64_t pre = 0, tot = 0;
-#pragma unroll
-            for (int q = 0; q < QW; q++) {
-                const uint64_t o = 32 * q + lane, idx = r0 + warp * per_w + o;
-                if (it > 0 && o < per_w && idx < r1) {
-#ifdef SZX_EXP_NOWAIT
-                    rv[q] |= 1ull << 63;
-#endif
-                    while (!(rv[q] >> 63)) {  // a lagging CTA has not published yet
-                        __nanosleep(32);
-                        rv[q] = ld_relaxed(&p.status_c[idx]);
-                    }
-                    const uint64_t val = rv[q] & ~(1ull << 63);
-                    tot += val;
-                    pre += idx < t_prev ? val : 0;
-                }
-            }
-            pre = warp_sum64(pre);
-            tot = warp_sum64(tot);
-            if (lane == 0) { s_pre[warp] = pre; s_tot[warp] = tot; }
-        }
-        __syncthreads();  // #2: this tile staged; the previous tile's round sizes summed
-        if (it > 0) {
-            uint64_t pre = 0, tot = 0;
-#pragma unroll
-            for (int w = 0; w < 8; w++) { pre += s_pre[w]; tot += s_tot[w]; }
-            copy_out(stg0 + ((it + C::NSTG - 1) % C::NSTG) * C::STG + 16, t_prev, run_base + pre, tb_prev);
-            run_base += tot;
-        }
-        tb_pp = tb_prev;
-        tb_prev = Tb;
-        t_prev = t;
-        if (tn >= ntiles) break;
-        t = tn;
-        cur = nxt;
-    }
-    // drain: the last tile of this CTA (its round's sizes, then copy-out)
-    {
-        const uint64_t G = gridDim.x;
-        const uint64_t r0 = t_prev / G * G;
-        uint64_t pre = 0;
-        for (uint64_t idx = r0 + threadIdx.x; idx < t_prev; idx += 256) {
-            uint64_t v = ld_relaxed(&p.status_c[idx]);
-            while (!(v >> 63)) {
-                __nanosleep(32);
-                v = ld_relaxed(&p.status_c[idx]);
-            }
-            pre += v & ~(1ull << 63);
-        }
-        pre = warp_sum64(pre);
-        __syncthreads();  // s_pre may still be read by the last iteration
-        if (lane == 0) s_pre[warp] = pre;
-        __syncthreads();
-        pre = 0;
-#pragma unroll
-        for (int w = 0; w < 8; w++) pre += s_pre[w];
-        copy_out(stg0 + (it % C::NSTG) * C::STG + 16, t_prev, run_base + pre, tb_prev);
     }
 }
 
