@@ -544,6 +544,11 @@ __device__ inline int guard_R(const T (&xv)[VPL], int cnt, T mu, int R, double e
 // Full float32 blocks of b = 128 (4 values per lane) with a FINAL R (the guard
 // has run): shifted words, lead codes and the per-value mid-byte counts, all
 // branch-free.  Identical output to encode_block/encode_known_R.
+// min(3, leading zero bytes of d): the 2-bit lead code (R6) in 4 instructions
+__device__ __forceinline__ uint32_t lead_bytes3(uint32_t d) {
+    return (uint32_t)__clz(d | 0xFFu) >> 3;
+}
+
 struct Lane4 {
     uint32_t u[4];      // shifted words
     uint32_t leads;     // 2-bit codes, LSB-first
@@ -562,7 +567,7 @@ __device__ __forceinline__ void lane_encode_f32x4(const float (&xv)[4], float mu
     uint32_t leads = 0, msum = 0;
 #pragma unroll
     for (int i = 0; i < 4; i++) {
-        const uint32_t L = umin_(3u, (uint32_t)__clz(e.u[i] ^ prev) >> 3);
+        const uint32_t L = lead_bytes3(e.u[i] ^ prev);
         prev = e.u[i];
         leads |= L << (2 * i);
         msum += req - umin_(L, req);
@@ -585,7 +590,7 @@ __device__ __forceinline__ uint32_t lane_msum_f32x4(const float (&xv)[4], float 
     uint32_t msum = 0;
 #pragma unroll
     for (int i = 0; i < 4; i++) {
-        const uint32_t L = umin_(3u, (uint32_t)__clz(u[i] ^ prev) >> 3);
+        const uint32_t L = lead_bytes3(u[i] ^ prev);
         prev = u[i];
         msum += req - umin_(L, req);
     }
@@ -627,9 +632,11 @@ __device__ __forceinline__ void lane_pack_f32x4(const Lane4& e, int R, uint32_t 
         const uint32_t lo = c0 | __funnelshift_lc(0u, c1, 8 * m0);
         const uint32_t hi = __funnelshift_lc(c1, 0u, 8 * m0);
         const uint32_t sh = 8 * (a & 3u), wa = a & ~3u;
-        red_or_nz(wa, lo << sh);
-        red_or_nz(wa + 4, __funnelshift_l(lo, hi, sh));
-        red_or_nz(wa + 8, __funnelshift_l(hi, 0u, sh));
+        // at most 8 bytes + 3 of misalignment: the third word is rarely needed
+        red_or_s(wa, lo << sh);
+        red_or_s(wa + 4, __funnelshift_l(lo, hi, sh));
+        const uint32_t w2 = __funnelshift_l(hi, 0u, sh);
+        if (w2) red_or_s(wa + 8, w2);
         a += m0 + m1;
     }
 }

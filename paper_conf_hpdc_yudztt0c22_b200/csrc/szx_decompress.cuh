@@ -111,7 +111,7 @@ __device__ inline uint64_t cta_scan256(uint64_t v, uint64_t* agg, uint64_t* s_w 
 #define SZX_EXP 0
 #endif
 #ifndef SZX_STCS
-#define SZX_STCS 0
+#define SZX_STCS 1
 #endif
 #ifndef SZX_ROT
 #define SZX_ROT 0
