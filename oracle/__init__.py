@@ -78,6 +78,10 @@ def lib():
         L.orc_shift_for.argtypes = [c_int]
         L.orc_identical_leading_bytes.restype = c_int
         L.orc_identical_leading_bytes.argtypes = [u64, u64, c_int]
+        L.orc_quality.restype = c_int
+        L.orc_quality.argtypes = [vp, vp, c_int, u64, vp]
+        L.orc_shift_overhead.restype = c_int
+        L.orc_shift_overhead.argtypes = [vp, u64, vp, vp]
         _lib = L
     return _lib
 
@@ -242,3 +246,44 @@ def shift_for(R: int) -> int:
 
 def identical_leading_bytes(prev: int, cur: int, W: int) -> int:
     return int(lib().orc_identical_leading_bytes(prev, cur, W))
+
+
+def quality(x: np.ndarray, xr: np.ndarray) -> dict:
+    """Max abs error (Formula 1's quantity), SSE / MSE, finite value range and
+    PSNR (Formula 7) of a reconstruction xr of x."""
+    x = np.ascontiguousarray(x).reshape(-1)
+    xr = np.ascontiguousarray(xr, dtype=x.dtype).reshape(-1)
+    assert x.size == xr.size
+    q = np.zeros(4, np.float64)
+    r = lib().orc_quality(x.ctypes.data if x.size else None, xr.ctypes.data if xr.size else None,
+                          _dtype_code(x), x.size, q.ctypes.data)
+    if r < 0:
+        raise ValueError(f"orc_quality failed: {r}")
+    return _quality_dict(q, x.size)
+
+
+def _quality_dict(q, n: int) -> dict:
+    maxe, sse, dmin, dmax = (float(v) for v in q)
+    mse = sse / n if n else 0.0
+    rng = dmax - dmin
+    if mse == 0.0:
+        psnr = float("inf")
+    elif not np.isfinite(mse) or not rng > 0:
+        psnr = float("-inf")
+    else:
+        psnr = 20.0 * np.log10(rng / np.sqrt(mse))
+    return dict(max_abs_err=maxe, sse=sse, mse=mse, dmin=dmin, dmax=dmax, psnr=float(psnr))
+
+
+def shift_overhead(stream: np.ndarray, x: np.ndarray) -> dict:
+    """Formula 6: necessary bits under Solution C (stored) and
+    Solution A/B, and the overhead relative to the stream size."""
+    stream = np.ascontiguousarray(stream, dtype=np.uint8)
+    x = np.ascontiguousarray(x).reshape(-1)
+    out = np.zeros(2, np.uint64)
+    r = lib().orc_shift_overhead(stream.ctypes.data, stream.size, x.ctypes.data if x.size else None,
+                                 out.ctypes.data)
+    if r < 0:
+        raise ValueError(f"orc_shift_overhead failed: {r}")
+    bc, bb = int(out[0]), int(out[1])
+    return dict(bits_C=bc, bits_B=bb, overhead=(bc - bb) / 8.0 / stream.size)
