@@ -152,6 +152,36 @@ int szx_decompress_async(const void* d_in, uint64_t in_bytes, const szx_header_t
                          void* d_out, uint64_t out_capacity_bytes, void* d_ws, uint64_t ws_bytes,
                          int32_t* d_status, void* stream);
 
+/* ------------------------------------------- reconstruction quality */
+
+/* Decompress (as szx_decompress: SZX1 or SZXC) and, fused into the same
+ * kernel, compare every reconstructed value with the original d_ref (device,
+ * 16-byte aligned, n values of the stream's dtype, laid out like d_out).
+ * h_qual (host, 4 doubles) receives:
+ *   [0] max |x - x'| -- the quantity Formula 1 bounds, in
+ *       double; identical bit patterns count 0, otherwise a NaN on either
+ *       side counts +Inf;
+ *   [1] sum (x - x')^2 in double (MSE = [1] / n; summation order is not
+ *       fixed, so it is reproducible to rounding only);
+ *   [2], [3] min and max of the finite x (+Inf / -Inf if none).
+ * PSNR = 20 log10(([3] - [2]) / sqrt([1] / n)) (Formula 7).
+ * Blocking.  Returns n or SZX_EINVAL / SZX_ENOSPC / SZX_ECORRUPT /
+ * SZX_ECUDA / SZX_ENOMEM. */
+int64_t szx_decompress_quality(const void* d_in, uint64_t in_bytes, const void* d_ref, void* d_out,
+                               uint64_t out_capacity_bytes, double* h_qual, void* stream);
+
+/* Non-blocking variant for one SZX1 stream (arguments as
+ * szx_decompress_async).  d_qual (device, 4 x uint64, caller-owned) is
+ * initialised on the stream and receives the raw accumulators
+ * {max-error bits, sum of squares (double bits), order key of the min,
+ * complemented order key of the max}; szx_quality_finish converts a host
+ * copy of them into the 4 doubles above. */
+int szx_decompress_quality_async(const void* d_in, uint64_t in_bytes, const szx_header_t* h,
+                                 const void* d_ref, void* d_out, uint64_t out_capacity_bytes,
+                                 void* d_ws, uint64_t ws_bytes, uint64_t* d_qual, int32_t* d_status,
+                                 void* stream);
+void szx_quality_finish(const uint64_t* raw4, double* out4);
+
 /* ------------------------------------------------ end-to-end host buffers */
 
 /* Compress host data h_in into host buffer h_out (capacity out_capacity):

@@ -4,13 +4,14 @@ Public API (all GPU; no CPU fallback):
     compress(x, eb, mode="rel", block_size=128) -> uint8 CUDA tensor (the stream)
     decompress(stream) -> float32/float64 CUDA tensor
     decompress_blocks(stream, first_block, n_blocks) -> the values of a block range
+    decompress_quality(stream, ref) -> (values, max error / MSE / PSNR), fused into the decoder
     compress_host / decompress_host  -- end to end through host buffers
     Codec                            -- preallocated buffers, non-blocking calls
     dist                             -- block-range sharding over torch.distributed (NCCL)
 """
 from .szx import (ABS, F32, F64, REL, Codec, Header, SZxError, compress, compress_bound,  # noqa: F401
-                  compress_host, decompress, decompress_blocks, decompress_host, launch_count, read_header,
+                  compress_host, decompress, decompress_blocks, decompress_host, decompress_quality, launch_count, read_header,
                   set_r_bias, timing_enable, timing_read, timing_reset, workspace_bytes)
 
-__all__ = ["compress", "decompress", "decompress_blocks", "compress_host", "decompress_host", "Codec", "read_header",
+__all__ = ["compress", "decompress", "decompress_blocks", "decompress_quality", "compress_host", "decompress_host", "Codec", "read_header",
            "compress_bound", "workspace_bytes", "SZxError", "ABS", "REL", "F32", "F64"]

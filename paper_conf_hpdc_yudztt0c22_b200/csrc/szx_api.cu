@@ -221,6 +221,7 @@ void set_smem_attrs() {
     carve(k_zscan<Traits<T>::W>);
     carve(k_enc_write<T, VPL>);
     carve(k_decode_w<T, VPL>);
+    carve(k_decode_w<T, VPL, true>);
     cudaFuncSetAttribute(k_enc_write<T, VPL>, cudaFuncAttributeMaxDynamicSharedMemorySize, WriteCfg<T, VPL>::SMEM);
     cudaFuncSetAttribute(k_enc_size<T, VPL>, cudaFuncAttributeMaxDynamicSharedMemorySize, SizeCfg<T, VPL>::SMEM);
 
@@ -381,7 +382,8 @@ int parse_header(const uint8_t* b, uint64_t nbytes, szx_header_t* h) {
 // whose element 0 is the first value of block kb0.
 int enqueue_decompress(const void* d_in, uint64_t in_bytes, const szx_header_t* h, void* d_out,
                        uint64_t cap, void* d_ws, uint64_t ws_bytes, int32_t** d_err_out, cudaStream_t s,
-                       uint64_t kb0 = 0, uint64_t kb1 = UINT64_MAX) {
+                       uint64_t kb0 = 0, uint64_t kb1 = UINT64_MAX, const void* d_ref = nullptr,
+                       uint64_t* d_qual = nullptr) {
     if (!d_in || !aligned16(d_in) || !h) return SZX_EINVAL;
     if (h->dtype > 1 || !block_ok(h->block_size) || h->n > kMaxN) return SZX_EINVAL;
     if (in_bytes < kHeaderBytes) return SZX_ECORRUPT;
@@ -393,6 +395,7 @@ int enqueue_decompress(const void* d_in, uint64_t in_bytes, const szx_header_t* 
     const uint64_t n_out = e1 - e0;
     if (cap < W * n_out) return SZX_ENOSPC;
     if (n_out && (!d_out || !aligned16(d_out))) return SZX_EINVAL;
+    if (d_ref && (!aligned16(d_ref) || !d_qual)) return SZX_EINVAL;
     DLayout L = dlayout(h->n, h->block_size);
     if (!d_ws || !aligned16(d_ws)) return SZX_EINVAL;
     if (ws_bytes < L.total) return SZX_ENOSPC;
@@ -422,26 +425,34 @@ int enqueue_decompress(const void* d_in, uint64_t in_bytes, const szx_header_t* 
     // the kernels index the output by stream element; shift the base so that
     // element e0 lands on d_out[0] (only elements of [e0, e1) are stored)
     const uintptr_t ybase = reinterpret_cast<uintptr_t>(d_out) - W * e0;
+    if (d_ref) {
+        p.ref = reinterpret_cast<const void*>(reinterpret_cast<uintptr_t>(d_ref) - W * e0);
+        p.qual = d_qual;
+    }
     dispatch((szx_dtype_t)h->dtype, h->block_size, [&](auto tag, auto vpl) {
         using T = decltype(tag);
         constexpr int V = decltype(vpl)::value;
         set_smem_attrs<T, V>();
         // persistent, co-resident grid (index phase, grid barrier, then one
         // warp per 32-block tile)
-        static int occ = 0;
-        if (!occ) {
-            cudaFuncSetAttribute(k_decode_w<T, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, DecWCfg<T, V>::SMEM);
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_decode_w<T, V>, 256, DecWCfg<T, V>::SMEM);
-            if (occ <= 0) occ = 4;
-        }
-        uint64_t grid = cdiv(p.nWi, 8);
-        const uint64_t cap = (uint64_t)sm_count() * occ;
-        if (grid > cap) grid = cap;
-        if (grid > kMaxDecodeGrid) grid = kMaxDecodeGrid;
-        launch("k_decode", s, [&] {
-            launch_pdl(k_decode_w<T, V>, dim3((unsigned)grid), dim3(256), DecWCfg<T, V>::SMEM, s, p, in,
-                       reinterpret_cast<T*>(ybase));
-        });
+        auto go = [&](auto kern, int& occ, const char* name) {
+            if (!occ) {
+                cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, DecWCfg<T, V>::SMEM);
+                cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, 256, DecWCfg<T, V>::SMEM);
+                if (occ <= 0) occ = 2;
+            }
+            uint64_t grid = cdiv(p.nWi, 8);
+            const uint64_t gcap = (uint64_t)sm_count() * occ;
+            if (grid > gcap) grid = gcap;
+            if (grid > kMaxDecodeGrid) grid = kMaxDecodeGrid;
+            launch(name, s, [&] {
+                launch_pdl(kern, dim3((unsigned)grid), dim3(256), DecWCfg<T, V>::SMEM, s, p, in,
+                           reinterpret_cast<T*>(ybase));
+            });
+        };
+        static int occ = 0, occ_q = 0;
+        if (d_ref) go(k_decode_w<T, V, true>, occ_q, "k_decode_q");
+        else go(k_decode_w<T, V>, occ, "k_decode");
     });
     return cudaGetLastError() == cudaSuccess ? SZX_OK : SZX_ECUDA;
 }
@@ -516,8 +527,28 @@ int parse_parts(const void* d_in, uint64_t in_bytes, cudaStream_t s, std::vector
 // (each with its own workspace slice), then one synchronisation reads all
 // status words.  ranged: block indices are global over the container, which
 // requires every part to start on a block boundary of one common block size.
+// Quality accumulators {max err bits, sse, dkey(min), ~dkey(max)} -> doubles
+// {max |x - x'|, sum (x - x')^2, min finite x, max finite x}.
+void qual_finish(const uint64_t* raw, double* out) {
+    memcpy(&out[0], &raw[0], 8);
+    memcpy(&out[1], &raw[1], 8);
+    const uint64_t a = raw[2], b = ~raw[3];
+    const uint64_t ba = dkey_inv(a), bb = dkey_inv(b);
+    double dmn, dmx;
+    memcpy(&dmn, &ba, 8);
+    memcpy(&dmx, &bb, 8);
+    out[2] = raw[2] == ~0ull ? INFINITY : dmn;
+    out[3] = raw[3] == ~0ull ? -INFINITY : dmx;
+}
+
+int qual_init(uint64_t* d_qual, cudaStream_t s) {
+    if (cudaMemsetAsync(d_qual, 0, 16, s) != cudaSuccess) return SZX_ECUDA;
+    if (cudaMemsetAsync(d_qual + 2, 0xFF, 16, s) != cudaSuccess) return SZX_ECUDA;
+    return SZX_OK;
+}
+
 int64_t decode_range(const void* d_in, uint64_t in_bytes, uint64_t g0, uint64_t g1, void* d_out, uint64_t cap,
-                     cudaStream_t s, bool ranged) {
+                     cudaStream_t s, bool ranged, const void* d_ref = nullptr, double* h_qual = nullptr) {
     if (!d_in || in_bytes < 64) return SZX_ECORRUPT;
     if (!have_device()) return SZX_ECUDA;
     std::vector<Part> parts;
@@ -535,7 +566,11 @@ int64_t decode_range(const void* d_in, uint64_t in_bytes, uint64_t g0, uint64_t 
     const uint64_t e0 = ranged ? g0 * b : 0, e1 = ranged ? std::min(total, g1 * b) : total;
     const uint64_t n_out = e1 > e0 ? e1 - e0 : 0;
     if (cap < W * n_out) return SZX_ENOSPC;
-    if (n_out == 0) return 0;
+    if (d_ref && (!h_qual || !aligned16(d_ref))) return SZX_EINVAL;
+    if (n_out == 0) {
+        if (h_qual) { const uint64_t z[4] = {0, 0, ~0ull, ~0ull}; qual_finish(z, h_qual); }
+        return 0;
+    }
     // per part: local block range, output position, workspace slice
     struct Job { size_t i; uint64_t kb0, kb1, out_el, ws_off; };
     std::vector<Job> jobs;
@@ -556,16 +591,22 @@ int64_t decode_range(const void* d_in, uint64_t in_bytes, uint64_t g0, uint64_t 
     }
     void* ws = nullptr;
     keep_pool_memory();
+    const uint64_t q_off = wsb;
+    wsb += 32;
     if (cudaMallocAsync(&ws, std::max<uint64_t>(wsb, 16), s) != cudaSuccess) { cudaGetLastError(); return SZX_ENOMEM; }
+    uint64_t* d_qual = reinterpret_cast<uint64_t*>(static_cast<uint8_t*>(ws) + q_off);
     std::vector<int32_t*> errs;
     int64_t r = 0;
+    if (d_ref) r = qual_init(d_qual, s);
     for (const Job& j : jobs) {
         const Part& pt = parts[j.i];
         int32_t* d_err = nullptr;
         const uint64_t wsz = al16(szx_decompress_workspace_bytes(&pt.h));
         rc = enqueue_decompress(static_cast<const uint8_t*>(d_in) + pt.off, pt.len, &pt.h,
                                 static_cast<uint8_t*>(d_out) + W * j.out_el, cap - W * j.out_el,
-                                static_cast<uint8_t*>(ws) + j.ws_off, wsz, &d_err, s, j.kb0, j.kb1);
+                                static_cast<uint8_t*>(ws) + j.ws_off, wsz, &d_err, s, j.kb0, j.kb1,
+                                d_ref ? static_cast<const uint8_t*>(d_ref) + W * j.out_el : nullptr,
+                                d_ref ? d_qual : nullptr);
         if (rc) { r = rc; break; }
         errs.push_back(d_err);
     }
@@ -574,6 +615,11 @@ int64_t decode_range(const void* d_in, uint64_t in_bytes, uint64_t g0, uint64_t 
         int32_t e = 0;
         if (cudaMemcpy(&e, errs[i], 4, cudaMemcpyDeviceToHost) != cudaSuccess) r = SZX_ECUDA;
         else if (e) r = e;
+    }
+    if (r == 0 && d_ref) {
+        uint64_t raw[4];
+        if (cudaMemcpy(raw, d_qual, 32, cudaMemcpyDeviceToHost) != cudaSuccess) r = SZX_ECUDA;
+        else qual_finish(raw, h_qual);
     }
     timing_resolve();
     cudaFreeAsync(ws, s);
@@ -667,6 +713,31 @@ int64_t szx_decompress_ws(const void* d_in, uint64_t in_bytes, void* d_out, uint
 int64_t szx_decompress(const void* d_in, uint64_t in_bytes, void* d_out, uint64_t cap, void* stream) {
     return decode_range(d_in, in_bytes, 0, UINT64_MAX, d_out, cap, static_cast<cudaStream_t>(stream), false);
 }
+
+int64_t szx_decompress_quality(const void* d_in, uint64_t in_bytes, const void* d_ref, void* d_out, uint64_t cap,
+                               double* h_qual, void* stream) {
+    if (!d_ref || !h_qual) return SZX_EINVAL;
+    return decode_range(d_in, in_bytes, 0, UINT64_MAX, d_out, cap, static_cast<cudaStream_t>(stream), false, d_ref,
+                        h_qual);
+}
+
+int szx_decompress_quality_async(const void* d_in, uint64_t in_bytes, const szx_header_t* h, const void* d_ref,
+                                 void* d_out, uint64_t cap, void* d_ws, uint64_t ws_bytes, uint64_t* d_qual,
+                                 int32_t* d_status, void* stream) {
+    if (!have_device()) return SZX_ECUDA;
+    if (!d_ref || !d_qual) return SZX_EINVAL;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    int rc = qual_init(d_qual, s);
+    if (rc) return rc;
+    int32_t* d_err = nullptr;
+    rc = enqueue_decompress(d_in, in_bytes, h, d_out, cap, d_ws, ws_bytes, &d_err, s, 0, UINT64_MAX, d_ref, d_qual);
+    if (rc) return rc;
+    if (d_status && d_status != d_err)
+        if (cudaMemcpyAsync(d_status, d_err, 4, cudaMemcpyDeviceToDevice, s) != cudaSuccess) return SZX_ECUDA;
+    return SZX_OK;
+}
+
+void szx_quality_finish(const uint64_t* raw, double* out) { qual_finish(raw, out); }
 
 int64_t szx_decompress_blocks(const void* d_in, uint64_t in_bytes, uint64_t first_block, uint64_t n_blocks,
                               void* d_out, uint64_t cap, void* stream) {

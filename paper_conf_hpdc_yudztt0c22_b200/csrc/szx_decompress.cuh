@@ -45,6 +45,64 @@ struct DPlan {
     uint32_t* ncpre;           // [nW]      nonconstant index of each tile's first block
     uint64_t* tbase;           // [nW + 1]  payload offset of each tile (tbase[nW] = total)
     int32_t* err;              // 0 ok, else SZX_ECORRUPT
+    // quality variant only: the original values, indexed
+    // like y, and the accumulators {max |x-x'| (double bits), sum (x-x')^2
+    // (double), dkey(min finite x), ~dkey(max finite x)}, initialised by the host
+    const void* ref;
+    uint64_t* qual;
+};
+
+// Per-thread reconstruction-quality accumulators (the fused max-error / PSNR
+// of SURVEY 8(f) row 1): Formula 1's max |x - x'| and Formula 7's MSE and
+// value range, with the oracle's definitions
+// (identical bits -> 0, a NaN otherwise -> +Inf; range over finite x).
+struct QualAcc {
+    double maxe = 0.0, sse = 0.0;
+    uint64_t kmn = ~0ull, kmx = 0ull;
+    template <typename T>
+    __device__ __forceinline__ void add(T x, T xr) {
+        using TR = Traits<T>;
+        const double dx = (double)x, dr = (double)xr;
+        double e = fabs(__dsub_rn(dx, dr));
+        e = (dx != dx || dr != dr) ? __longlong_as_double(0x7FF0000000000000ll) : e;
+        e = TR::bits(x) == TR::bits(xr) ? 0.0 : e;
+        maxe = e > maxe ? e : maxe;
+        sse = __dadd_rn(sse, __dmul_rn(e, e));
+        const uint64_t k = dkey((uint64_t)__double_as_longlong(dx));
+        const bool fin = fabs(dx) < __longlong_as_double(0x7FF0000000000000ll);
+        kmn = fin && k < kmn ? k : kmn;
+        kmx = fin && k > kmx ? k : kmx;
+    }
+    // 16-byte chunks of decoded values against the same chunks of the original
+    template <typename T, int NV>
+    __device__ __forceinline__ void add16(const uint4* ref, const uint4 (&v)[NV]) {
+#pragma unroll
+        for (int q = 0; q < NV; q++) {
+            const uint4 r = ld_stream16(ref + q);
+            const T* a = reinterpret_cast<const T*>(&r);
+            const T* b = reinterpret_cast<const T*>(&v[q]);
+#pragma unroll
+            for (int i = 0; i < 16 / (int)sizeof(T); i++) add<T>(a[i], b[i]);
+        }
+    }
+    // warp reduction, then one set of atomics per warp
+    __device__ void flush(uint64_t* q) {
+        uint64_t m = (uint64_t)__double_as_longlong(maxe);
+        double ss = sse;
+#pragma unroll
+        for (int o = 16; o; o >>= 1) {
+            const uint64_t m2 = __shfl_xor_sync(0xffffffffu, m, o);
+            m = m2 > m ? m2 : m;
+            ss = __dadd_rn(ss, __shfl_xor_sync(0xffffffffu, ss, o));
+        }
+        const uint64_t a = warp_min(kmn), b = warp_max(kmx);
+        if ((threadIdx.x & 31) == 0) {
+            atomicMax((unsigned long long*)&q[0], (unsigned long long)m);  // e >= 0: bit order = value order
+            atomicAdd(reinterpret_cast<double*>(&q[1]), ss);
+            atomicMin((unsigned long long*)&q[2], (unsigned long long)a);
+            atomicMin((unsigned long long*)&q[3], (unsigned long long)~b);
+        }
+    }
 };
 
 // Stream facts read from the 64-byte header in device memory, validated
@@ -545,7 +603,7 @@ struct TileMeta {
     U mul;              // lane j: mu of block j
 };
 
-template <typename T, int VPL>
+template <typename T, int VPL, bool QUAL = false>
 __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint8_t* __restrict__ in, T* __restrict__ y) {
     using TR = Traits<T>;
     using U = typename TR::U;
@@ -558,6 +616,8 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
     constexpr int QB = B * W / 16;    // 16-byte chunks per block
     extern __shared__ __align__(16) uint8_t dsm[];
     __shared__ uint64_t s_w[32];
+    QualAcc qa;
+    const T* __restrict__ ref = static_cast<const T*>(p.ref);
     pdl_wait();
     pdl_trigger();
     const DHdr hd = read_dheader<W>(in, p);
@@ -626,6 +686,9 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
                 for (int q = 0; q < VPL; q++) v[q] = TR::from(mb);
 #pragma unroll
                 for (int q = 0; q < NV; q++) st_out16(yq + j * QB + q, reinterpret_cast<const uint4*>(v)[q]);
+                if constexpr (QUAL)
+                    qa.add16<T, NV>(reinterpret_cast<const uint4*>(ref + t * TB * B + lane * VPL) + j * QB,
+                                    reinterpret_cast<const uint4(&)[NV]>(v));
             }
             t = tn;
             word = wn;
@@ -734,6 +797,9 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
             }
 #pragma unroll
             for (int q = 0; q < NV; q++) st_out16(yq + j * QB + q, reinterpret_cast<const uint4*>(v)[q]);
+            if constexpr (QUAL)
+                qa.add16<T, NV>(reinterpret_cast<const uint4*>(ref + t * TB * B + lane * VPL) + j * QB,
+                                reinterpret_cast<const uint4(&)[NV]>(v));
         }
     };
     // the partial last tile: generic decoder, straight from global memory
@@ -761,6 +827,12 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
                 }
             }
             store_lane<T, VPL>(y, p.n, k, lane, v);
+            if constexpr (QUAL) {
+                const uint64_t first = k * B + (uint64_t)lane * VPL;
+#pragma unroll
+                for (int i = 0; i < VPL; i++)
+                    if (first + i < p.n) qa.add<T>(ref[first + i], v[i]);
+            }
         }
     };
 
@@ -831,6 +903,7 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
         nc_loop();
         if (SZX_SWITCH & 1) fill_loop();
     }
+    if constexpr (QUAL) qa.flush(p.qual);
 }
 
 }  // namespace szx

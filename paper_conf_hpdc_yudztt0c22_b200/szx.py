@@ -8,6 +8,7 @@ the library or a CUDA device is missing, every call raises.
 from __future__ import annotations
 
 import ctypes
+import math
 import os
 import struct
 from dataclasses import dataclass
@@ -62,6 +63,10 @@ def lib() -> ctypes.CDLL:
         "szx_decompress_async": (i32, [vp, u64, ctypes.POINTER(_Header), vp, u64, vp, u64, vp, vp]),
         "szx_compress_host": (i64, [vp, i32, u64, i32, dbl, u32, vp, u64, vp]),
         "szx_decompress_host": (i64, [vp, u64, vp, u64, vp]),
+        "szx_decompress_quality": (i64, [vp, u64, vp, vp, u64, vp, vp]),
+        "szx_decompress_quality_async": (i32, [vp, u64, ctypes.POINTER(_Header), vp, vp, u64, vp, u64, vp, vp,
+                                               vp]),
+        "szx_quality_finish": (None, [vp, vp]),
         "szx_local_range": (i32, [vp, i32, u64, u32, vp, vp, u64, vp]),
         "szx_compress_shard_async": (i32, [vp, i32, u64, i32, dbl, vp, u32, vp, u64, vp, u64, vp, vp]),
         "szx_timing_enable": (None, [i32]),
@@ -83,7 +88,8 @@ def lib() -> ctypes.CDLL:
 EXPORTED = ["szx_compress_bound", "szx_compress_workspace_bytes", "szx_decompress_workspace_bytes",
             "szx_compress", "szx_compress_ws", "szx_compress_async", "szx_read_header",
             "szx_decompress", "szx_decompress_blocks", "szx_decompress_ws", "szx_decompress_async", "szx_compress_host",
-            "szx_decompress_host", "szx_local_range", "szx_compress_shard_async",
+            "szx_decompress_host", "szx_decompress_quality", "szx_decompress_quality_async",
+            "szx_quality_finish", "szx_local_range", "szx_compress_shard_async",
             "szx_timing_enable", "szx_timing_reset", "szx_timing_read", "szx_launch_count",
             "szx_debug_set_r_bias", "szx_strerror"]
 
@@ -227,6 +233,39 @@ def decompress_blocks(s: torch.Tensor, first_block: int, n_blocks: int, out: tor
     return out[:r]
 
 
+def _quality_dict(q, n: int) -> dict:
+    maxe, sse, dmin, dmax = (float(v) for v in q)
+    mse = sse / n if n else 0.0
+    rng = dmax - dmin
+    if mse == 0.0:
+        psnr = math.inf
+    elif not math.isfinite(mse) or not rng > 0:
+        psnr = -math.inf
+    else:
+        psnr = 20.0 * math.log10(rng / math.sqrt(mse))
+    return dict(max_abs_err=maxe, sse=sse, mse=mse, dmin=dmin, dmax=dmax, psnr=psnr)
+
+
+def decompress_quality(s: torch.Tensor, ref: torch.Tensor, out: torch.Tensor | None = None, stream=None):
+    """Decompress and, fused into the decode kernel, measure the reconstruction against the
+    original ``ref``: returns (values, {max_abs_err, sse, mse, dmin, dmax, psnr}) -- Formula 1's
+    max error and Formula 7's PSNR."""
+    _require_cuda(s)
+    _require_cuda(ref)
+    n, dt = _container_info(s)
+    tdt = torch.float32 if dt == F32 else torch.float64
+    ref = ref.contiguous().view(-1)
+    if ref.numel() != n or ref.dtype != tdt:
+        raise ValueError(f"reference must hold {n} {tdt} values")
+    if out is None:
+        out = torch.empty(max(n, 1), dtype=tdt, device=s.device)
+    q = (ctypes.c_double * 4)()
+    r = lib().szx_decompress_quality(s.data_ptr(), s.numel(), ref.data_ptr() if n else None, out.data_ptr(),
+                                     out.numel() * out.element_size(), q, _stream(stream))
+    _check(r, "szx_decompress_quality")
+    return out[:n], _quality_dict(list(q), n)
+
+
 def compress_host(x, eb: float, mode="rel", block_size: int = 128, out=None, stream=None):
     """End-to-end compress of a HOST tensor (ideally pinned) through the C ABI's host entry point.
     Returns a uint8 CPU tensor view of the stream."""
@@ -305,6 +344,26 @@ class Codec:
                                         y.numel() * y.element_size(), self.dws.data_ptr(), self.dws.numel(),
                                         self.d_status.data_ptr(), _stream(stream))
         _check(rc, "szx_decompress_async")
+
+    def decompress_quality_async(self, s: torch.Tensor, h: Header, y: torch.Tensor, ref: torch.Tensor,
+                                 stream=None):
+        """decompress_async with the fused quality accumulators (read with ``quality()``)."""
+        need = int(lib().szx_decompress_workspace_bytes(ctypes.byref(h._c)))
+        if self.dws is None or self.dws.numel() < need:
+            self.dws = torch.empty(max(need, 16), dtype=torch.uint8, device=self.device)
+        if getattr(self, "d_qual", None) is None:
+            self.d_qual = torch.zeros(4, dtype=torch.int64, device=self.device)
+        rc = lib().szx_decompress_quality_async(s.data_ptr(), s.numel(), ctypes.byref(h._c), ref.data_ptr(),
+                                                y.data_ptr(), y.numel() * y.element_size(), self.dws.data_ptr(),
+                                                self.dws.numel(), self.d_qual.data_ptr(),
+                                                self.d_status.data_ptr(), _stream(stream))
+        _check(rc, "szx_decompress_quality_async")
+
+    def quality(self) -> dict:
+        raw = self.d_qual.cpu().numpy()
+        q = (ctypes.c_double * 4)()
+        lib().szx_quality_finish(raw.ctypes.data, q)
+        return _quality_dict(list(q), self.n)
 
 
 def timing_enable(on: bool = True):
