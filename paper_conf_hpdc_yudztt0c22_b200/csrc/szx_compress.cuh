@@ -689,6 +689,62 @@ __global__ void __launch_bounds__(256) k_enc_size(const T* __restrict__ x, Plan 
         const uint32_t mk = gv ? p.nclist[gi] : 0u;
         const U mmu = gv ? ncmu[gi] : U(0);
         const uint32_t mrec = gv ? p.ncR[gi] : 0u;
+        if constexpr (sizeof(T) == 4 && VPL == 4) {
+            // fast path: 32 full float32 blocks (the list is in block order, so
+            // the last one decides): no per-block bounds or tail tests, and z_k /
+            // R collected in lane l for one coalesced store per 32 blocks
+            if (c1 - g0 >= 32 && __shfl_sync(0xffffffffu, mk, 31) < nBfull) {
+                auto issue_f = [&](int b) {
+                    const uint32_t st = sbuf + (b & 1) * C::NB * C::BW;
+#pragma unroll
+                    for (int j = 0; j < C::NB; j++) {
+                        const uint32_t k = __shfl_sync(0xffffffffu, mk, b * C::NB + j);
+                        cp_async16(st + j * C::BW + lane * 16, x + (uint64_t)k * B + lane * 4);
+                    }
+                    cp_async_commit();
+                };
+                uint32_t zr = 0, rr = 0;
+                issue_f(0);
+#pragma unroll 1
+                for (int b = 0; b < 32 / C::NB; b++) {
+                    if (b + 1 < 32 / C::NB) {
+                        issue_f(b + 1);
+                        cp_async_wait<1>();
+                    } else {
+                        cp_async_wait<0>();
+                    }
+                    __syncwarp();
+                    const uint32_t st = sbuf + (b & 1) * C::NB * C::BW;
+#pragma unroll
+                    for (int j = 0; j < C::NB; j += 2) {
+                        const int l = b * C::NB + j;
+                        float x0[4], x1[4];
+                        reinterpret_cast<uint4*>(x0)[0] = lds_u128(st + j * C::BW + lane * 16);
+                        reinterpret_cast<uint4*>(x1)[0] = lds_u128(st + (j + 1) * C::BW + lane * 16);
+                        const float mu0 = __uint_as_float(__shfl_sync(0xffffffffu, (uint32_t)mmu, l));
+                        const float mu1 = __uint_as_float(__shfl_sync(0xffffffffu, (uint32_t)mmu, l + 1));
+                        const uint32_t rec0 = __shfl_sync(0xffffffffu, mrec, l);
+                        const uint32_t rec1 = __shfl_sync(0xffffffffu, mrec, l + 1);
+                        int R0 = (int)(rec0 & 0x7F), R1 = (int)(rec1 & 0x7F);
+                        if (!(rec0 & rec1 & 0x80)) {  // a block whose R2 check was not proven away
+                            if (!(rec0 & 0x80)) R0 = guard_R<float, 4>(x0, 4, mu0, R0, eb);
+                            if (!(rec1 & 0x80)) R1 = guard_R<float, 4>(x1, 4, mu1, R1, eb);
+                        }
+                        const uint32_t z0 = 33u + warp_sum(lane_msum_f32x4(x0, mu0, R0));
+                        const uint32_t z1 = 33u + warp_sum(lane_msum_f32x4(x1, mu1, R1));
+                        zr = lane == l ? z0 : zr;
+                        rr = lane == l ? (uint32_t)R0 : rr;
+                        zr = lane == l + 1 ? z1 : zr;
+                        rr = lane == l + 1 ? (uint32_t)R1 : rr;
+                    }
+                    __syncwarp();
+                }
+                zsize[gi] = (uint16_t)zr;
+                p.ncR[gi] = (uint8_t)rr;
+                if (rr >= 32u) mus[mk] = 0;  // raw (NaN, Formula 4 or escalation): mu = +0 (R15)
+                continue;
+            }
+        }
         const int nbat = (int)((umin64(32, c1 - g0) + C::NB - 1) / C::NB);
         auto issue = [&](int b) {
             const uint32_t st = sbuf + (b & 1) * C::NB * C::BW;
@@ -932,10 +988,12 @@ __global__ void __launch_bounds__(256) k_enc_write(const T* __restrict__ x, Plan
     const U mmu = mv ? ncmu[ncw + lane] : U(0);
     const uint32_t mR = mv ? p.ncR[ncw + lane] : 0u;
     const uint32_t sin = smem_u32(stg) + C::STG + warp * C::BPW * C::BW;
+    // whole tile of full blocks (the list is in block order: the tile's last block decides)
+    const bool tfull = (t + 1) * C::TB <= nnc && p.nclist[(t + 1) * C::TB - 1] < nBfull;
 #pragma unroll
     for (int j = 0; j < C::BPW; j++) {
         const uint32_t k = __shfl_sync(0xffffffffu, mk, j);
-        if (ncw + j < nnc && k < nBfull) {
+        if (tfull || (ncw + j < nnc && k < nBfull)) {
             const T* src = x + (uint64_t)k * C::B + lane * VPL;
 #pragma unroll
             for (int q = 0; q < C::QV; q++) cp_async16(sin + j * C::BW + (lane * C::QV + q) * 16, src + q * (16 / W));
@@ -954,6 +1012,24 @@ __global__ void __launch_bounds__(256) k_enc_write(const T* __restrict__ x, Plan
     }
     cp_async_wait<0>();
     __syncthreads();
+    if constexpr (sizeof(T) == 4 && VPL == 4) {
+        if (tfull) {  // branch-free body: every block of the tile is a full float32 block
+#pragma unroll
+            for (int j = 0; j < C::BPW; j++) {
+                const int bi = warp * C::BPW + j;
+                const uint32_t zo = __shfl_sync(0xffffffffu, zincl - zl, bi);
+                const float cmu = __uint_as_float(__shfl_sync(0xffffffffu, (uint32_t)mmu, j));
+                const int R = (int)__shfl_sync(0xffffffffu, mR, j);
+                float xv[4];
+                reinterpret_cast<uint4*>(xv)[0] = lds_u128(sin + j * C::BW + lane * 16);
+                Lane4 e;
+                lane_encode_f32x4(xv, cmu, R, e);
+                const uint32_t incl = warp_incl_scan(e.msum);
+                lane_pack_f32x4(e, R, incl - e.msum, smem_u32(stg) + sb + zo);
+            }
+            goto copy_out;
+        }
+    }
 #pragma unroll 1
     for (int j = 0; j < C::BPW; j++) {
         const int bi = warp * C::BPW + j;
@@ -986,6 +1062,7 @@ __global__ void __launch_bounds__(256) k_enc_write(const T* __restrict__ x, Plan
             pack_red<T, VPL>(u, lc, cnt, len, smem_u32(stg) + sb + zo);
         }
     }
+copy_out:
     __syncthreads();
     // copy the staged tile payload to global memory with 16-byte stores
     uint8_t* g0 = out + off_pl + base;
@@ -996,11 +1073,18 @@ __global__ void __launch_bounds__(256) k_enc_write(const T* __restrict__ x, Plan
         const uint4 v = *reinterpret_cast<const uint4*>(stg + 16 * ch);
         if (a >= a0 && a + 16 <= E) {
             *reinterpret_cast<uint4*>(a) = v;
-        } else {
-            const uint8_t* vb = reinterpret_cast<const uint8_t*>(&v);
+        } else {  // a boundary chunk shared with the neighbouring tiles: whole words, then bytes
+            const uint32_t vw[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
-            for (int q = 0; q < 16; q++)
-                if (a + q >= a0 && a + q < E) *reinterpret_cast<uint8_t*>(a + q) = vb[q];
+            for (int q = 0; q < 4; q++) {
+                const uintptr_t aw = a + 4 * q;
+                if (aw >= a0 && aw + 4 <= E) {
+                    *reinterpret_cast<uint32_t*>(aw) = vw[q];
+                } else if (aw + 4 > a0 && aw < E) {
+                    for (int c = 0; c < 4; c++)
+                        if (aw + c >= a0 && aw + c < E) *reinterpret_cast<uint8_t*>(aw + c) = (uint8_t)(vw[q] >> (8 * c));
+                }
+            }
         }
     }
 }

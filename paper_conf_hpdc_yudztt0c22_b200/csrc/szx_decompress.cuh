@@ -776,20 +776,19 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
                                (uint32_t)(reinterpret_cast<uintptr_t>(pl + m.base + sg.off0) & 15) - sg.off0;
         uint4* yq = reinterpret_cast<uint4*>(y + t * TB * B + lane * VPL);
         const uint32_t rm = rmask(t);
-        // blocks whose rank lies in [r0, r1): clear the set bits below r0 and from r1 on
-        uint32_t sel = m.word;
-        for (uint32_t r = 0; r < sg.r0; r++) sel &= sel - 1;
-        uint32_t keep = sel;
-        for (uint32_t r = sg.r0; r < sg.r1; r++) keep &= keep - 1;
-        sel &= ~keep;
-        uint32_t r = sg.r0;
+        // blocks whose rank lies in [r0, r1), restricted to the requested range;
+        // lane j holds block j's payload offset and size (one shuffle each per segment)
+        const uint32_t rank = __popc(m.word & ((1u << lane) - 1u));
+        const bool insg = ((m.word >> lane) & 1u) && rank >= sg.r0 && rank < sg.r1;
+        const uint32_t sel = __ballot_sync(0xffffffffu, insg) & rm;
+        const uint32_t offl = __shfl_sync(0xffffffffu, z.zincl - z.zl, rank);
+        const uint32_t zzl = __shfl_sync(0xffffffffu, z.zl, rank);
 #pragma unroll 1
-        for (uint32_t bits = (SZX_EXP & 2) ? 0u : sel; bits; bits &= bits - 1, r++) {
+        for (uint32_t bits = (SZX_EXP & 2) ? 0u : sel; bits; bits &= bits - 1) {
             const int j = __ffs(bits) - 1;
-            const uint32_t off = __shfl_sync(0xffffffffu, z.zincl - z.zl, r);
-            const uint32_t zz = __shfl_sync(0xffffffffu, z.zl, r);
+            const uint32_t off = __shfl_sync(0xffffffffu, offl, j);
+            const uint32_t zz = __shfl_sync(0xffffffffu, zzl, j);
             const T mu = TR::from(__shfl_sync(0xffffffffu, m.mul, j));
-            if (!((rm >> j) & 1u)) continue;
             T v[VPL];
             if (!decode_full_g<T, VPL>(SrcS{sbase + off}, zz, mu, v)) {
                 if (lane == 0) set_corrupt(p.err);
