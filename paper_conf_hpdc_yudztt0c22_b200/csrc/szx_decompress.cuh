@@ -174,6 +174,9 @@ __device__ inline uint64_t cta_scan256(uint64_t v, uint64_t* agg, uint64_t* s_w 
 #ifndef SZX_ROT
 #define SZX_ROT 0
 #endif
+#ifndef SZX_PAIR
+#define SZX_PAIR 1   // float32 b = 128: two blocks per warp, a half-warp each
+#endif
 constexpr int kIndexChunk = 256;
 
 // Copy zs[i0, i0 + cnt) (cnt <= 32 * kIndexChunk) into shared memory with
@@ -492,6 +495,89 @@ __device__ __forceinline__ bool decode_full_f32x4(const Src src, uint32_t z, flo
     return true;
 }
 
+// ---- two float32 blocks of b = 128 per warp: a half-warp per block, 8 values
+// per lane.  Same arithmetic as decode_full_f32x4 (Fig. 10's five steps), but
+// every per-lane step -- R / code parsing, the mid-byte scan, the lead-byte
+// map scan, the z check -- is paid once per 8 values instead of once per 4.
+// Inclusive prefix sum within 16-lane segments (predicated by shfl's in-segment flag)
+template <int O>
+__device__ __forceinline__ uint32_t shfl_up_add16(uint32_t v) {
+    asm volatile(
+        "{\n\t.reg .u32 t;\n\t.reg .pred p;\n\t"
+        "shfl.sync.up.b32 t|p, %0, %1, 0x1000, -1;\n\t"
+        "@p add.u32 %0, %0, t;\n\t}"
+        : "+r"(v)
+        : "n"(O));
+    return v;
+}
+// Half-warp h decodes the block whose payload starts at shared address a
+// (z bytes); returns false (for the whole half) on a malformed block.
+__device__ __forceinline__ bool decode_half_f32x8(uint32_t a, uint32_t z, float mu, float (&out)[8]) {
+    const int sl = threadIdx.x & 15;
+    const uint32_t R = lds_u8(a);
+    const bool bad = R < 9u || R > 32u;
+    const bool raw = R >= 32u;
+    const uint32_t s = raw ? 0u : ((8u - (R & 7u)) & 7u);
+    const uint32_t req = bad ? 4u : (R + s) >> 3;       // 2..4 kept bytes
+    const uint32_t leads = lds_u8(a + 1 + 2 * sl) | (lds_u8(a + 2 + 2 * sl) << 8);
+    uint32_t m[8], nm[8];
+#pragma unroll
+    for (int i = 0; i < 8; i++) {
+        const uint32_t L = (leads >> (2 * i)) & 3u;
+        const uint32_t copy = L < req ? L : req;
+        m[i] = req - copy;
+        nm[i] = 0xFFFFFFFFu >> (8 * copy);      // bytes NOT copied from the previous value
+    }
+    const uint32_t m01 = m[0] + m[1], m23 = m[2] + m[3], m45 = m[4] + m[5];
+    const uint32_t msum = m01 + m23 + m45 + m[6] + m[7];
+    uint32_t incl = shfl_up_add16<1>(msum);
+    incl = shfl_up_add16<2>(incl);
+    incl = shfl_up_add16<4>(incl);
+    incl = shfl_up_add16<8>(incl);
+    const uint32_t tot = __shfl_sync(0xffffffffu, incl, 15, 16);
+    const bool ok = !bad && 33u + tot == z;
+    const uint32_t o = 33u + incl - msum;
+    uint32_t ra[2], rb[2], rc[2], rd[2];
+    run_load_s<2>(a + o, ra);
+    run_load_s<2>(a + o + m01, rb);
+    run_load_s<2>(a + o + m01 + m23, rc);
+    run_load_s<2>(a + o + m01 + m23 + m45, rd);
+    const uint32_t drop = 8u * (4u - req);
+    auto lowmask = [](uint32_t mm) { return ~__funnelshift_lc(0u, 0xFFFFFFFFu, 8u * mm); };
+    uint32_t own[8];
+    own[0] = (ra[0] & lowmask(m[0])) << drop;
+    own[1] = (__funnelshift_rc(ra[0], ra[1], 8u * m[0]) & lowmask(m[1])) << drop;
+    own[2] = (rb[0] & lowmask(m[2])) << drop;
+    own[3] = (__funnelshift_rc(rb[0], rb[1], 8u * m[2]) & lowmask(m[3])) << drop;
+    own[4] = (rc[0] & lowmask(m[4])) << drop;
+    own[5] = (__funnelshift_rc(rc[0], rc[1], 8u * m[4]) & lowmask(m[5])) << drop;
+    own[6] = (rd[0] & lowmask(m[6])) << drop;
+    own[7] = (__funnelshift_rc(rd[0], rd[1], 8u * m[6]) & lowmask(m[7])) << drop;
+    // lane map c -> (c & M) | D, then its exclusive scan within the half
+    uint32_t cM = ~(nm[0] | nm[1] | nm[2] | nm[3] | nm[4] | nm[5] | nm[6] | nm[7]);
+    uint32_t cD = own[0];
+#pragma unroll
+    for (int i = 1; i < 8; i++) cD = (cD & ~nm[i]) | own[i];
+#pragma unroll
+    for (int d = 1; d < 16; d <<= 1) {
+        const uint32_t pM = __shfl_up_sync(0xffffffffu, cM, d, 16);
+        const uint32_t pD = __shfl_up_sync(0xffffffffu, cD, d, 16);
+        // lanes below d in the half get their own map back: composing a map
+        // with itself leaves it unchanged
+        cD = (pD & cM) | cD;
+        cM = pM & cM;
+    }
+    uint32_t prev = __shfl_up_sync(0xffffffffu, cD, 1, 16);
+    prev = sl == 0 ? 0u : prev;
+#pragma unroll
+    for (int i = 0; i < 8; i++) {
+        const uint32_t w = (prev & ~nm[i]) | own[i];
+        prev = w;
+        out[i] = raw ? __uint_as_float(w) : __fadd_rn(__uint_as_float(w << s), mu);
+    }
+    return ok;
+}
+
 // decode_full with the payload in global memory
 template <typename T, int VPL, typename Src>
 __device__ inline bool decode_full_g(const Src src, uint32_t z, T mu, T (&out)[VPL]) {
@@ -783,6 +869,42 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
         const uint32_t sel = __ballot_sync(0xffffffffu, insg) & rm;
         const uint32_t offl = __shfl_sync(0xffffffffu, z.zincl - z.zl, rank);
         const uint32_t zzl = __shfl_sync(0xffffffffu, z.zl, rank);
+#if SZX_PAIR
+        if constexpr (sizeof(T) == 4 && VPL == 4) {
+            // two blocks per iteration, a half-warp each (the second half idles
+            // on the last block of an odd count)
+            const int h = lane >> 4, hl = lane & 15;
+            float* yb = reinterpret_cast<float*>(y) + t * TB * B + hl * 8;
+#pragma unroll 1
+            for (uint32_t bits = sel; bits;) {
+                const int j0 = __ffs(bits) - 1;
+                bits &= bits - 1;
+                const bool two = bits != 0;
+                const int j1 = two ? __ffs(bits) - 1 : j0;
+                bits &= bits - 1;
+                const int jh = h ? j1 : j0;
+                const uint32_t off = __shfl_sync(0xffffffffu, offl, jh);
+                const uint32_t zz = __shfl_sync(0xffffffffu, zzl, jh);
+                const float mu = __uint_as_float(__shfl_sync(0xffffffffu, (uint32_t)m.mul, jh));
+                float v[8];
+                const bool ok = decode_half_f32x8(sbase + off, zz, mu, v);
+                if (h == 0 || two) {
+                    if (!ok) {
+                        if (hl == 0) set_corrupt(p.err);
+                    } else {
+                        uint4* q = reinterpret_cast<uint4*>(yb + jh * B);
+                        st_out16(q, reinterpret_cast<const uint4*>(v)[0]);
+                        st_out16(q + 1, reinterpret_cast<const uint4*>(v)[1]);
+                        if constexpr (QUAL) {
+                            const uint4* rq = reinterpret_cast<const uint4*>(ref + t * TB * B + jh * B + hl * 8);
+                            qa.add16<T, 2>(rq, reinterpret_cast<const uint4(&)[2]>(v));
+                        }
+                    }
+                }
+            }
+            return;
+        }
+#endif
 #pragma unroll 1
         for (uint32_t bits = (SZX_EXP & 2) ? 0u : sel; bits; bits &= bits - 1) {
             const int j = __ffs(bits) - 1;
