@@ -31,6 +31,10 @@
 
 #include "szx_device.cuh"
 
+#ifndef SZX_WPAIR
+#define SZX_WPAIR 1   // size and write passes: two float32 blocks per warp, a half-warp each
+#endif
+
 namespace szx {
 
 struct Plan {
@@ -597,6 +601,105 @@ __device__ __forceinline__ uint32_t lane_msum_f32x4(const float (&xv)[4], float 
     return msum;
 }
 
+// ---- half-warp variants (8 values per lane, a block per 16 lanes): the
+// write pass encodes two blocks per warp instruction stream
+struct Lane8 {
+    uint32_t u[8];      // shifted words
+    uint32_t leads;     // 2-bit codes of the 8 values, LSB-first (16 bits)
+    uint32_t msum;      // mid-bytes of this lane
+};
+__device__ __forceinline__ void lane_encode_f32x8(const float (&xv)[8], float mu, int R, Lane8& e) {
+    const int hl = threadIdx.x & 15;
+    const bool raw = R >= 32;
+    const uint32_t s = raw ? 0u : ((8u - ((uint32_t)R & 7u)) & 7u);
+    const uint32_t req = ((uint32_t)R + s) >> 3;
+#pragma unroll
+    for (int i = 0; i < 8; i++)
+        e.u[i] = (raw ? __float_as_uint(xv[i]) : __float_as_uint(__fsub_rn(xv[i], mu))) >> s;
+    uint32_t prev = __shfl_up_sync(0xffffffffu, e.u[7], 1, 16);
+    prev = hl == 0 ? 0u : prev;
+    uint32_t leads = 0, msum = 0;
+#pragma unroll
+    for (int i = 0; i < 8; i++) {
+        const uint32_t L = lead_bytes3(e.u[i] ^ prev);
+        prev = e.u[i];
+        leads |= L << (2 * i);
+        msum += req - umin_(L, req);
+    }
+    e.leads = leads;
+    e.msum = msum;
+}
+// inclusive prefix sum within 16-lane segments
+template <int O>
+__device__ __forceinline__ uint32_t shfl_up_add16c(uint32_t v) {
+    asm volatile(
+        "{\n\t.reg .u32 t;\n\t.reg .pred p;\n\t"
+        "shfl.sync.up.b32 t|p, %0, %1, 0x1000, -1;\n\t"
+        "@p add.u32 %0, %0, t;\n\t}"
+        : "+r"(v)
+        : "n"(O));
+    return v;
+}
+__device__ __forceinline__ uint32_t half_incl_scan(uint32_t v) {
+    v = shfl_up_add16c<1>(v);
+    v = shfl_up_add16c<2>(v);
+    v = shfl_up_add16c<4>(v);
+    return shfl_up_add16c<8>(v);
+}
+__device__ inline void red_or_s(uint32_t a, uint32_t v);
+// Pack a full float32 block held by a half-warp into the zeroed staging area at dst.
+__device__ __forceinline__ void lane_pack_f32x8(const Lane8& e, int R, uint32_t mexcl, uint32_t dst) {
+    const int hl = threadIdx.x & 15;
+    if (hl == 0) red_or_s(dst & ~3u, (uint32_t)R << (8 * (dst & 3u)));
+    {   // this lane's two code bytes (they may straddle a word)
+        const uint32_t a = dst + 1 + 2 * hl, sh = 8 * (a & 3u);
+        red_or_s(a & ~3u, e.leads << sh);
+        const uint32_t w1 = __funnelshift_l(e.leads, 0u, sh);
+        if (w1) red_or_s((a & ~3u) + 4, w1);
+    }
+    const bool raw = R >= 32;
+    const uint32_t s = raw ? 0u : ((8u - ((uint32_t)R & 7u)) & 7u);
+    const uint32_t req = ((uint32_t)R + s) >> 3;
+    const uint32_t drop = 8u * (4u - req);
+    uint32_t a = dst + 33 + mexcl;
+#pragma unroll
+    for (int h = 0; h < 4; h++) {
+        const uint32_t m0 = req - umin_((e.leads >> (4 * h)) & 3u, req);
+        const uint32_t m1 = req - umin_((e.leads >> (4 * h + 2)) & 3u, req);
+        const uint32_t c0 = (e.u[2 * h] >> drop) & ~__funnelshift_lc(0u, 0xFFFFFFFFu, 8 * m0);
+        const uint32_t c1 = (e.u[2 * h + 1] >> drop) & ~__funnelshift_lc(0u, 0xFFFFFFFFu, 8 * m1);
+        const uint32_t lo = c0 | __funnelshift_lc(0u, c1, 8 * m0);
+        const uint32_t hi = __funnelshift_lc(c1, 0u, 8 * m0);
+        const uint32_t sh = 8 * (a & 3u), wa = a & ~3u;
+        red_or_s(wa, lo << sh);
+        red_or_s(wa + 4, __funnelshift_l(lo, hi, sh));
+        const uint32_t w2 = __funnelshift_l(hi, 0u, sh);
+        if (w2) red_or_s(wa + 8, w2);
+        a += m0 + m1;
+    }
+}
+
+// Mid-bytes of this lane's 8 values (size pass, half-warp per block)
+__device__ __forceinline__ uint32_t lane_msum_f32x8(const float (&xv)[8], float mu, int R) {
+    const int hl = threadIdx.x & 15;
+    const bool raw = R >= 32;
+    const uint32_t s = raw ? 0u : ((8u - ((uint32_t)R & 7u)) & 7u);
+    const uint32_t req = ((uint32_t)R + s) >> 3;
+    uint32_t u[8];
+#pragma unroll
+    for (int i = 0; i < 8; i++) u[i] = (raw ? __float_as_uint(xv[i]) : __float_as_uint(__fsub_rn(xv[i], mu))) >> s;
+    uint32_t prev = __shfl_up_sync(0xffffffffu, u[7], 1, 16);
+    prev = hl == 0 ? 0u : prev;
+    uint32_t msum = 0;
+#pragma unroll
+    for (int i = 0; i < 8; i++) {
+        const uint32_t L = lead_bytes3(u[i] ^ prev);
+        prev = u[i];
+        msum += req - umin_(L, req);
+    }
+    return msum;
+}
+
 // OR v into shared word a unless v == 0 (predicated, no branch)
 __device__ __forceinline__ void red_or_nz(uint32_t a, uint32_t v) {
 #ifdef SZX_EXP_STS
@@ -715,6 +818,43 @@ __global__ void __launch_bounds__(256) k_enc_size(const T* __restrict__ x, Plan 
                     }
                     __syncwarp();
                     const uint32_t st = sbuf + (b & 1) * C::NB * C::BW;
+#if SZX_WPAIR
+                    // two blocks at once, a half-warp each (8 values per lane)
+#pragma unroll
+                    for (int j = 0; j < C::NB; j += 2) {
+                        const int l = b * C::NB + j;
+                        const int h = lane >> 4, hl = lane & 15;
+                        float xv[8];
+                        reinterpret_cast<uint4*>(xv)[0] = lds_u128(st + (j + h) * C::BW + hl * 32);
+                        reinterpret_cast<uint4*>(xv)[1] = lds_u128(st + (j + h) * C::BW + hl * 32 + 16);
+                        const float mu = __uint_as_float(__shfl_sync(0xffffffffu, (uint32_t)mmu, l + h));
+                        const uint32_t rec = __shfl_sync(0xffffffffu, mrec, l + h);
+                        int R = (int)(rec & 0x7F);
+                        if (!__all_sync(0xffffffffu, (rec & 0x80) != 0)) {
+                            // a block whose R2 check was not proven away: full-warp guard per block
+                            float x0[4], x1[4];
+                            reinterpret_cast<uint4*>(x0)[0] = lds_u128(st + j * C::BW + lane * 16);
+                            reinterpret_cast<uint4*>(x1)[0] = lds_u128(st + (j + 1) * C::BW + lane * 16);
+                            const uint32_t rec0 = __shfl_sync(0xffffffffu, mrec, l);
+                            const uint32_t rec1 = __shfl_sync(0xffffffffu, mrec, l + 1);
+                            const float mu0 = __uint_as_float(__shfl_sync(0xffffffffu, (uint32_t)mmu, l));
+                            const float mu1 = __uint_as_float(__shfl_sync(0xffffffffu, (uint32_t)mmu, l + 1));
+                            int R0 = (int)(rec0 & 0x7F), R1 = (int)(rec1 & 0x7F);
+                            if (!(rec0 & 0x80)) R0 = guard_R<float, 4>(x0, 4, mu0, R0, eb);
+                            if (!(rec1 & 0x80)) R1 = guard_R<float, 4>(x1, 4, mu1, R1, eb);
+                            R = h ? R1 : R0;
+                        }
+                        const uint32_t ms = lane_msum_f32x8(xv, mu, R);
+                        const uint32_t z0 = 33u + warp_sum(h ? 0u : ms);
+                        const uint32_t z1 = 33u + warp_sum(h ? ms : 0u);
+                        const uint32_t R0 = __shfl_sync(0xffffffffu, (uint32_t)R, 0);
+                        const uint32_t R1 = __shfl_sync(0xffffffffu, (uint32_t)R, 16);
+                        zr = lane == l ? z0 : zr;
+                        rr = lane == l ? R0 : rr;
+                        zr = lane == l + 1 ? z1 : zr;
+                        rr = lane == l + 1 ? R1 : rr;
+                    }
+#else
 #pragma unroll
                     for (int j = 0; j < C::NB; j += 2) {
                         const int l = b * C::NB + j;
@@ -737,6 +877,7 @@ __global__ void __launch_bounds__(256) k_enc_size(const T* __restrict__ x, Plan 
                         zr = lane == l + 1 ? z1 : zr;
                         rr = lane == l + 1 ? (uint32_t)R1 : rr;
                     }
+#endif
                     __syncwarp();
                 }
                 zsize[gi] = (uint16_t)zr;
@@ -1014,6 +1155,26 @@ __global__ void __launch_bounds__(256) k_enc_write(const T* __restrict__ x, Plan
     __syncthreads();
     if constexpr (sizeof(T) == 4 && VPL == 4) {
         if (tfull) {  // branch-free body: every block of the tile is a full float32 block
+#if SZX_WPAIR
+            // two blocks per step, a half-warp each (8 values per lane)
+            const int h = lane >> 4, hl = lane & 15;
+#pragma unroll
+            for (int q = 0; q < C::BPW / 2; q++) {
+                const int j = 2 * q + h;
+                const int bi = warp * C::BPW + j;
+                const uint32_t zo = __shfl_sync(0xffffffffu, zincl - zl, bi);
+                const float cmu = __uint_as_float(__shfl_sync(0xffffffffu, (uint32_t)mmu, j));
+                const int R = (int)__shfl_sync(0xffffffffu, mR, j);
+                float xv[8];
+                reinterpret_cast<uint4*>(xv)[0] = lds_u128(sin + j * C::BW + hl * 32);
+                reinterpret_cast<uint4*>(xv)[1] = lds_u128(sin + j * C::BW + hl * 32 + 16);
+                Lane8 e;
+                lane_encode_f32x8(xv, cmu, R, e);
+                const uint32_t incl = half_incl_scan(e.msum);
+                lane_pack_f32x8(e, R, incl - e.msum, smem_u32(stg) + sb + zo);
+            }
+            goto copy_out;
+#endif
 #pragma unroll
             for (int j = 0; j < C::BPW; j++) {
                 const int bi = warp * C::BPW + j;
