@@ -601,6 +601,17 @@ __device__ __forceinline__ uint32_t lane_msum_f32x4(const float (&xv)[4], float 
     return msum;
 }
 
+// OR v into shared word a unless v == 0 (predicated, no branch)
+__device__ __forceinline__ void red_or_nz(uint32_t a, uint32_t v) {
+#ifdef SZX_EXP_STS
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %1, 0;\n\t@q st.shared.b32 [%0], %1;\n\t}"
+                 ::"r"(a), "r"(v) : "memory");
+#else
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %1, 0;\n\t@q red.shared.or.b32 [%0], %1;\n\t}"
+                 ::"r"(a), "r"(v) : "memory");
+#endif
+}
+
 // ---- half-warp variants (8 values per lane, a block per 16 lanes): the
 // write pass encodes two blocks per warp instruction stream
 struct Lane8 {
@@ -655,7 +666,7 @@ __device__ __forceinline__ void lane_pack_f32x8(const Lane8& e, int R, uint32_t 
         const uint32_t a = dst + 1 + 2 * hl, sh = 8 * (a & 3u);
         red_or_s(a & ~3u, e.leads << sh);
         const uint32_t w1 = __funnelshift_l(e.leads, 0u, sh);
-        if (w1) red_or_s((a & ~3u) + 4, w1);
+        red_or_nz((a & ~3u) + 4, w1);
     }
     const bool raw = R >= 32;
     const uint32_t s = raw ? 0u : ((8u - ((uint32_t)R & 7u)) & 7u);
@@ -673,8 +684,7 @@ __device__ __forceinline__ void lane_pack_f32x8(const Lane8& e, int R, uint32_t 
         const uint32_t sh = 8 * (a & 3u), wa = a & ~3u;
         red_or_s(wa, lo << sh);
         red_or_s(wa + 4, __funnelshift_l(lo, hi, sh));
-        const uint32_t w2 = __funnelshift_l(hi, 0u, sh);
-        if (w2) red_or_s(wa + 8, w2);
+        red_or_nz(wa + 8, __funnelshift_l(hi, 0u, sh));
         a += m0 + m1;
     }
 }
@@ -700,16 +710,6 @@ __device__ __forceinline__ uint32_t lane_msum_f32x8(const float (&xv)[8], float 
     return msum;
 }
 
-// OR v into shared word a unless v == 0 (predicated, no branch)
-__device__ __forceinline__ void red_or_nz(uint32_t a, uint32_t v) {
-#ifdef SZX_EXP_STS
-    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %1, 0;\n\t@q st.shared.b32 [%0], %1;\n\t}"
-                 ::"r"(a), "r"(v) : "memory");
-#else
-    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %1, 0;\n\t@q red.shared.or.b32 [%0], %1;\n\t}"
-                 ::"r"(a), "r"(v) : "memory");
-#endif
-}
 // Pack a full float32 block into a zeroed shared staging area at byte address
 // dst: [R][32 code bytes][mid-bytes].  Values are placed in pairs: the two
 // chunks (<= 8 bytes) are joined with funnel shifts and OR-ed in as at most
@@ -738,8 +738,7 @@ __device__ __forceinline__ void lane_pack_f32x4(const Lane4& e, int R, uint32_t 
         // at most 8 bytes + 3 of misalignment: the third word is rarely needed
         red_or_s(wa, lo << sh);
         red_or_s(wa + 4, __funnelshift_l(lo, hi, sh));
-        const uint32_t w2 = __funnelshift_l(hi, 0u, sh);
-        if (w2) red_or_s(wa + 8, w2);
+        red_or_nz(wa + 8, __funnelshift_l(hi, 0u, sh));
         a += m0 + m1;
     }
 }

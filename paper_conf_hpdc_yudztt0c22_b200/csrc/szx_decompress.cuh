@@ -518,46 +518,46 @@ __device__ __forceinline__ bool decode_half_f32x8(uint32_t a, uint32_t z, float 
     const bool bad = R < 9u || R > 32u;
     const bool raw = R >= 32u;
     const uint32_t s = raw ? 0u : ((8u - (R & 7u)) & 7u);
-    const uint32_t req = bad ? 4u : (R + s) >> 3;       // 2..4 kept bytes
+    const uint32_t r8 = bad ? 32u : (R + s);            // kept bits: 8 x (2..4 bytes)
+    const uint32_t drop = 32u - r8;
     const uint32_t leads = lds_u8(a + 1 + 2 * sl) | (lds_u8(a + 2 + 2 * sl) << 8);
-    uint32_t m[8], nm[8];
+    // per value, in bits: c8 = 8 x bytes copied from the previous value
+    // (min(lead, req), step 2), m8 = 8 x mid-bytes read (step 3); nm masks the
+    // bytes NOT copied
+    uint32_t m8[8], nm[8];
 #pragma unroll
     for (int i = 0; i < 8; i++) {
-        const uint32_t L = (leads >> (2 * i)) & 3u;
-        const uint32_t copy = L < req ? L : req;
-        m[i] = req - copy;
-        nm[i] = 0xFFFFFFFFu >> (8 * copy);      // bytes NOT copied from the previous value
+        const uint32_t c8 = umin((leads >> (2 * i) << 3) & 24u, r8);
+        m8[i] = r8 - c8;
+        nm[i] = 0xFFFFFFFFu >> c8;
     }
-    const uint32_t m01 = m[0] + m[1], m23 = m[2] + m[3], m45 = m[4] + m[5];
-    const uint32_t msum = m01 + m23 + m45 + m[6] + m[7];
+    const uint32_t b01 = m8[0] + m8[1], b23 = m8[2] + m8[3], b45 = m8[4] + m8[5];
+    const uint32_t msum = (b01 + b23 + b45 + m8[6] + m8[7]) >> 3;
     uint32_t incl = shfl_up_add16<1>(msum);
     incl = shfl_up_add16<2>(incl);
     incl = shfl_up_add16<4>(incl);
     incl = shfl_up_add16<8>(incl);
     const uint32_t tot = __shfl_sync(0xffffffffu, incl, 15, 16);
     const bool ok = !bad && 33u + tot == z;
-    const uint32_t o = 33u + incl - msum;
-    uint32_t ra[2], rb[2], rc[2], rd[2];
-    run_load_s<2>(a + o, ra);
-    run_load_s<2>(a + o + m01, rb);
-    run_load_s<2>(a + o + m01 + m23, rc);
-    run_load_s<2>(a + o + m01 + m23 + m45, rd);
-    const uint32_t drop = 8u * (4u - req);
-    auto lowmask = [](uint32_t mm) { return ~__funnelshift_lc(0u, 0xFFFFFFFFu, 8u * mm); };
-    uint32_t own[8];
-    own[0] = (ra[0] & lowmask(m[0])) << drop;
-    own[1] = (__funnelshift_rc(ra[0], ra[1], 8u * m[0]) & lowmask(m[1])) << drop;
-    own[2] = (rb[0] & lowmask(m[2])) << drop;
-    own[3] = (__funnelshift_rc(rb[0], rb[1], 8u * m[2]) & lowmask(m[3])) << drop;
-    own[4] = (rc[0] & lowmask(m[4])) << drop;
-    own[5] = (__funnelshift_rc(rc[0], rc[1], 8u * m[4]) & lowmask(m[5])) << drop;
-    own[6] = (rd[0] & lowmask(m[6])) << drop;
-    own[7] = (__funnelshift_rc(rd[0], rd[1], 8u * m[6]) & lowmask(m[7])) << drop;
+    const uint32_t o = a + 33u + incl - msum;
+    uint32_t r[4][2];
+    run_load_s<2>(o, r[0]);
+    run_load_s<2>(o + (b01 >> 3), r[1]);
+    run_load_s<2>(o + ((b01 + b23) >> 3), r[2]);
+    run_load_s<2>(o + ((b01 + b23 + b45) >> 3), r[3]);
+    // value i's mid-bytes moved to their place under the copied top bytes:
+    // sw & nm (the bytes below them are zero after the shift)
+    uint32_t sw[8];
+#pragma unroll
+    for (int q = 0; q < 4; q++) {
+        sw[2 * q] = r[q][0] << drop;
+        sw[2 * q + 1] = __funnelshift_rc(r[q][0], r[q][1], m8[2 * q]) << drop;
+    }
     // lane map c -> (c & M) | D, then its exclusive scan within the half
     uint32_t cM = ~(nm[0] | nm[1] | nm[2] | nm[3] | nm[4] | nm[5] | nm[6] | nm[7]);
-    uint32_t cD = own[0];
+    uint32_t cD = sw[0] & nm[0];
 #pragma unroll
-    for (int i = 1; i < 8; i++) cD = (cD & ~nm[i]) | own[i];
+    for (int i = 1; i < 8; i++) cD = (cD & ~nm[i]) | (sw[i] & nm[i]);
 #pragma unroll
     for (int d = 1; d < 16; d <<= 1) {
         const uint32_t pM = __shfl_up_sync(0xffffffffu, cM, d, 16);
@@ -571,7 +571,7 @@ __device__ __forceinline__ bool decode_half_f32x8(uint32_t a, uint32_t z, float 
     prev = sl == 0 ? 0u : prev;
 #pragma unroll
     for (int i = 0; i < 8; i++) {
-        const uint32_t w = (prev & ~nm[i]) | own[i];
+        const uint32_t w = (prev & ~nm[i]) | (sw[i] & nm[i]);
         prev = w;
         out[i] = raw ? __uint_as_float(w) : __fadd_rn(__uint_as_float(w << s), mu);
     }
