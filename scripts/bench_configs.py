@@ -55,11 +55,11 @@ def cases(box_full: bool):
     yield "box", "QMCPack-like 288x115x69x69 f64", lambda: synth.qmcpack_like(device="cuda"), [1e-4]
 
 
-def run_case(x: torch.Tensor, eb: float, iters: int, flush: torch.Tensor | None):
+def run_case(x: torch.Tensor, eb: float, iters: int, flush: torch.Tensor | None, b: int = 128):
     x = x.reshape(-1).contiguous()
     n = x.numel()
     W = x.element_size()
-    codec = szx.Codec(n, x.dtype, 128, device=x.device)
+    codec = szx.Codec(n, x.dtype, b, device=x.device)
     y = torch.empty_like(x)
     codec.compress_async(x, eb, "rel")
     S = codec.stream_bytes()
@@ -89,6 +89,20 @@ def run_case(x: torch.Tensor, eb: float, iters: int, flush: torch.Tensor | None)
             tc.append(ev[0].elapsed_time(ev[1]))
             td.append(ev[2].elapsed_time(ev[3]))
     assert int(codec.d_status.item()) == 0
+    # decompression with the fused quality accumulators (max error, PSNR)
+    tq = []
+    for i in range(3 + iters):
+        ev = [torch.cuda.Event(enable_timing=True) for _ in range(2)]
+        if flush is not None:
+            flush.fill_(i & 0xFF)
+        ev[0].record()
+        codec.decompress_quality_async(codec.out, h, y, x)
+        ev[1].record()
+        torch.cuda.synchronize()
+        if i >= 3:
+            tq.append(ev[0].elapsed_time(ev[1]))
+    q = codec.quality()
+    assert q["max_abs_err"] == err or n > 300_000_000, (q, err)
     # per-kernel breakdown (library events around each launch; separate pass)
     szx.timing_reset()
     szx.timing_enable(True)
@@ -106,7 +120,8 @@ def run_case(x: torch.Tensor, eb: float, iters: int, flush: torch.Tensor | None)
             "compress_ms": cms, "decompress_ms": dms,
             "compress_gbs": nb / cms / 1e6, "decompress_gbs": nb / dms / 1e6,
             "compress_hbm_frac": (2 * nb + S) / cms / 1e6 / pk, "decompress_hbm_frac": (S + nb) / dms / 1e6 / pk,
-            "kernels_ms": kt, "l2_flush": flush is not None}
+            "decompress_quality_ms": statistics.median(tq), "psnr": q["psnr"], "max_abs_err_fused": q["max_abs_err"],
+            "block": b, "kernels_ms": kt, "l2_flush": flush is not None}
 
 
 def main():
@@ -114,6 +129,7 @@ def main():
     ap.add_argument("--iters", type=int, default=20)
     ap.add_argument("--only", default="")
     ap.add_argument("--box-full", action="store_true")
+    ap.add_argument("--blocks", default="128", help="block sizes to sweep, e.g. 128,256 (SURVEY 8(f) row 2)")
     a = ap.parse_args()
     only = set(a.only.split(",")) if a.only else None
     l2 = torch.cuda.get_device_properties(0).L2_cache_size
@@ -125,9 +141,10 @@ def main():
         torch.cuda.synchronize()
         small = x.numel() * x.element_size() < 4 * l2
         for eb in ebs:
-            r = run_case(x, eb, a.iters, flush_buf if small else None)
-            r.update({"config": key, "workload": name, "eb_rel": eb, "peak_gbs": peak()})
-            print(json.dumps(r), flush=True)
+            for b in (int(v) for v in a.blocks.split(",")):
+                r = run_case(x, eb, a.iters, flush_buf if small else None, b)
+                r.update({"config": key, "workload": name, "eb_rel": eb, "peak_gbs": peak()})
+                print(json.dumps(r), flush=True)
         del x
         torch.cuda.empty_cache()
 
