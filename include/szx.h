@@ -194,6 +194,35 @@ int64_t szx_compress_host(const void* h_in, szx_dtype_t dt, uint64_t n, szx_ebmo
 int64_t szx_decompress_host(const void* h_in, uint64_t in_bytes, void* h_out,
                             uint64_t out_capacity_bytes, void* stream);
 
+/* ------------------------------------------------ dump / load through host memory */
+
+/* Dump a device array to host memory as an SZXC container of `parts`
+ * block-range shards (shard q: blocks [q nB / parts, (q+1) nB / parts),
+ * clipped to >= 1 block each; DESIGN.md s.8), the single-box analogue of the
+ * paper's data dumping experiment (Fig. 16).  One pass reads
+ * every shard's block statistics and local range (the REL bound is global,
+ * footnote 1); then shard q+1 compresses while shard q is copied
+ * device -> host on a second stream.  The container is byte-identical to
+ * szx_compress_shard_async of each shard with the global bound, assembled
+ * as in SURVEY Appendix A.
+ *   d_in   device, 16-byte aligned, n values of dt;
+ *   h_out  host (pinned for overlap; pageable works, serialised), h_cap bytes;
+ *   stream the compute stream (the copy stream is internal).
+ * Blocking.  Returns the container bytes, or SZX_EINVAL / SZX_ENOSPC (h_cap
+ * too small: the sum of the shard streams, not the bound, must fit) /
+ * SZX_ECUDA / SZX_ENOMEM.  Device scratch: the shards' workspaces plus two
+ * stream buffers of one shard's bound. */
+int64_t szx_dump_host(const void* d_in, szx_dtype_t dt, uint64_t n, szx_ebmode_t mode, double eb,
+                      uint32_t block_size, uint32_t parts, void* h_out, uint64_t h_cap, void* stream);
+
+/* Load an SZX1 stream or SZXC container held in host memory (h_in, pinned
+ * for overlap) into the device array d_out (16-byte aligned, >= n W bytes):
+ * shard q+1 is copied host -> device while shard q decodes (Fig. 10,
+ * P:L2321-2336).  Blocking.  Returns n, or SZX_ECORRUPT / SZX_ENOSPC /
+ * SZX_EINVAL / SZX_ECUDA / SZX_ENOMEM. */
+int64_t szx_load_host(const void* h_in, uint64_t in_bytes, void* d_out, uint64_t out_capacity_bytes,
+                      void* stream);
+
 /* ------------------------------------------------ sharded (multi-GPU) use */
 
 /* Pass 1 of a sharded compress: one read of the local shard that writes the

@@ -856,6 +856,231 @@ int szx_compress_shard_async(const void* d_in, szx_dtype_t dt, uint64_t n, szx_e
     return cudaGetLastError() == cudaSuccess ? SZX_OK : SZX_ECUDA;
 }
 
+
+// ------------------------------------------------------------ dump / load
+// Single-box analogue of the paper's data dumping / loading experiment
+// (Fig. 16): a device array goes to host memory as an SZXC
+// container of P block-range shards (DESIGN.md s.8), compression of shard
+// p+1 overlapping the device-to-host copy of shard p; loading copies shard
+// q+1 to the device while shard q decodes.
+
+__global__ void k_keys_min(const uint64_t* keys, uint32_t P, uint64_t* out) {
+    uint64_t a = ~0ull, c = ~0ull;
+    for (uint32_t i = 0; i < P; i++) {
+        a = keys[2 * i] < a ? keys[2 * i] : a;
+        c = keys[2 * i + 1] < c ? keys[2 * i + 1] : c;
+    }
+    out[0] = a;
+    out[1] = c;
+}
+
+namespace {
+struct DumpRes {  // device scratch (stream-ordered pool, kept between calls) and the copy stream / events
+    std::vector<void*> dev;
+    std::vector<cudaEvent_t> events;
+    cudaStream_t s = nullptr, s2 = nullptr;
+    ~DumpRes() {
+        if (s2) cudaStreamSynchronize(s2);
+        for (auto p : dev) cudaFreeAsync(p, s);
+        if (s) cudaStreamSynchronize(s);
+        for (auto e : events) cudaEventDestroy(e);
+        if (s2) cudaStreamDestroy(s2);
+    }
+    bool init(cudaStream_t st) {
+        s = st;
+        keep_pool_memory();
+        return cudaStreamCreateWithFlags(&s2, cudaStreamNonBlocking) == cudaSuccess;
+    }
+    void* dalloc(uint64_t bytes) {
+        void* p = nullptr;
+        if (cudaMallocAsync(&p, bytes ? bytes : 16, s) != cudaSuccess) { cudaGetLastError(); return nullptr; }
+        dev.push_back(p);
+        return p;
+    }
+    cudaEvent_t event() {
+        cudaEvent_t e = nullptr;
+        if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return nullptr;
+        events.push_back(e);
+        return e;
+    }
+};
+// pinned host slots for the shard sizes (per calling thread, grown on demand, kept)
+uint64_t* pinned_sizes(uint32_t P) {
+    thread_local uint64_t* buf = nullptr;
+    thread_local uint32_t cap = 0;
+    if (P > cap) {
+        if (buf) cudaFreeHost(buf);
+        buf = nullptr;
+        cap = 0;
+        if (cudaMallocHost(&buf, 8ull * P) != cudaSuccess) return nullptr;
+        cap = P;
+    }
+    return buf;
+}
+}  // namespace
+
+int64_t szx_dump_host(const void* d_in, szx_dtype_t dt, uint64_t n, szx_ebmode_t mode, double eb, uint32_t b,
+                      uint32_t parts, void* h_out, uint64_t h_cap, void* stream) {
+    int rc = check_compress_args(d_in, dt, n, mode, eb, b, d_in);
+    if (rc) return rc;
+    if (!h_out || parts == 0) return SZX_EINVAL;
+    if (!have_device()) return SZX_ECUDA;
+    const uint64_t W = wbytes(dt), nB = cdiv(n, b);
+    const uint32_t P = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(parts, std::max<uint64_t>(nB, 1)));
+    std::vector<uint64_t> e0(P), np(P);
+    uint64_t nmax = 0;
+    for (uint32_t q = 0; q < P; q++) {  // shard q: blocks [q nB / P, (q+1) nB / P)
+        const uint64_t b0 = nB * q / P, b1 = nB * (q + 1) / P;
+        e0[q] = b0 * b;
+        np[q] = std::min<uint64_t>(n, b1 * b) - std::min<uint64_t>(n, b0 * b);
+        nmax = std::max(nmax, np[q]);
+    }
+    const uint64_t head = 32 + 32ull * P;
+    if (h_cap < head) return SZX_ENOSPC;
+    DumpRes R;
+    if (!R.init(static_cast<cudaStream_t>(stream))) return SZX_ECUDA;
+    cudaStream_t s = R.s, s2 = R.s2;
+    std::vector<void*> ws(P);
+    std::vector<uint64_t> wsb(P);
+    for (uint32_t q = 0; q < P; q++) {
+        wsb[q] = std::max<uint64_t>(szx_compress_workspace_bytes(np[q], dt, b), 16);
+        if (!(ws[q] = R.dalloc(wsb[q]))) return SZX_ENOMEM;
+    }
+    uint64_t* keys = static_cast<uint64_t*>(R.dalloc(16ull * P + 16));
+    uint64_t* totals = static_cast<uint64_t*>(R.dalloc(8ull * P));
+    const uint64_t cap = szx_compress_bound(nmax, dt, b);
+    void* buf[2] = {R.dalloc(cap), R.dalloc(cap)};
+    uint64_t* hsz = pinned_sizes(P);
+    if (!hsz) return SZX_ENOMEM;
+    if (!keys || !totals || !buf[0] || !buf[1]) return SZX_ENOMEM;
+    const uint8_t* in = static_cast<const uint8_t*>(d_in);
+    // pass 1: block statistics and the local ranges of every shard, then the global range
+    for (uint32_t q = 0; q < P; q++) {
+        rc = szx_local_range(in + W * e0[q], dt, np[q], b, keys + 2 * q, ws[q], wsb[q], s);
+        if (rc) return rc;
+    }
+    uint64_t* gkeys = keys + 2 * P;
+    k_keys_min<<<1, 1, 0, s>>>(keys, P, gkeys);
+    // pass 2: shard q compresses on s while shard q-1 is copied out on s2
+    cudaEvent_t done[2] = {R.event(), R.event()}, copied[2] = {R.event(), R.event()};
+    uint8_t* ho = static_cast<uint8_t*>(h_out);
+    uint64_t pos = al16(head);
+    std::vector<uint64_t> off(P), sz(P);
+    auto copy_out = [&](uint32_t q) -> int {
+        if (cudaEventSynchronize(done[q & 1]) != cudaSuccess) return SZX_ECUDA;
+        sz[q] = hsz[q];
+        off[q] = pos;
+        if (pos + sz[q] > h_cap) return SZX_ENOSPC;
+        cudaStreamWaitEvent(s2, done[q & 1], 0);
+        if (cudaMemcpyAsync(ho + pos, buf[q & 1], sz[q], cudaMemcpyDeviceToHost, s2) != cudaSuccess) return SZX_ECUDA;
+        cudaEventRecord(copied[q & 1], s2);
+        const uint64_t end = pos + sz[q];
+        pos = q + 1 < P ? al16(end) : end;
+        if (pos > h_cap) return SZX_ENOSPC;
+        memset(ho + end, 0, pos - end);  // zero padding between shard streams
+        return SZX_OK;
+    };
+    for (uint32_t q = 0; q < P; q++) {
+        if (q >= 2) cudaStreamWaitEvent(s, copied[q & 1], 0);  // its buffer's previous copy is done
+        rc = szx_compress_shard_async(in + W * e0[q], dt, np[q], mode, eb, gkeys, b, buf[q & 1], cap, ws[q], wsb[q],
+                                      totals + q, s);
+        if (rc) return rc;
+        cudaMemcpyAsync(hsz + q, totals + q, 8, cudaMemcpyDeviceToHost, s);
+        cudaEventRecord(done[q & 1], s);
+        if (q >= 1 && (rc = copy_out(q - 1))) return rc;
+    }
+    if ((rc = copy_out(P - 1))) return rc;
+    if (cudaStreamSynchronize(s2) != cudaSuccess) return SZX_ECUDA;
+    // container header and shard table
+    memset(ho, 0, al16(head));
+    memcpy(ho, "SZXC", 4);
+    const uint32_t ver = 1, zero = 0;
+    memcpy(ho + 4, &ver, 4);
+    memcpy(ho + 8, &P, 4);
+    memcpy(ho + 12, &zero, 4);
+    memcpy(ho + 16, &n, 8);
+    for (uint32_t q = 0; q < P; q++) {
+        const uint64_t e[4] = {e0[q], np[q], off[q], sz[q]};
+        memcpy(ho + 32 + 32ull * q, e, 32);
+    }
+    timing_resolve();
+    return cudaGetLastError() == cudaSuccess ? (int64_t)pos : SZX_ECUDA;
+}
+
+int64_t szx_load_host(const void* h_in, uint64_t in_bytes, void* d_out, uint64_t cap, void* stream) {
+    if (!h_in || in_bytes < 64) return SZX_ECORRUPT;
+    if (!have_device()) return SZX_ECUDA;
+    const uint8_t* hb = static_cast<const uint8_t*>(h_in);
+    std::vector<Part> parts;
+    uint64_t total = 0;
+    if (memcmp(hb, "SZXC", 4) == 0) {
+        uint32_t P, ver;
+        memcpy(&ver, hb + 4, 4);
+        memcpy(&P, hb + 8, 4);
+        memcpy(&total, hb + 16, 8);
+        if (ver != 1 || P == 0 || 32 + 32ull * P > in_bytes) return SZX_ECORRUPT;
+        uint64_t expect = 0;
+        for (uint32_t i = 0; i < P; i++) {
+            uint64_t e[4];
+            memcpy(e, hb + 32 + 32ull * i, 32);
+            if (e[0] != expect || e[2] % 16 || e[2] > in_bytes || e[3] > in_bytes - e[2] || e[3] < 64)
+                return SZX_ECORRUPT;
+            Part pt;
+            if (parse_header(hb + e[2], e[3], &pt.h) || pt.h.n != e[1]) return SZX_ECORRUPT;
+            if (!parts.empty() && pt.h.dtype != parts[0].h.dtype) return SZX_ECORRUPT;
+            pt.off = e[2]; pt.len = e[3]; pt.first = e[0];
+            parts.push_back(pt);
+            expect += e[1];
+        }
+        if (expect != total) return SZX_ECORRUPT;
+    } else {
+        Part pt;
+        if (parse_header(hb, in_bytes, &pt.h)) return SZX_ECORRUPT;
+        pt.off = 0; pt.len = in_bytes; pt.first = 0;
+        parts.push_back(pt);
+        total = pt.h.n;
+    }
+    const uint64_t W = parts[0].h.dtype ? 8 : 4;
+    if (cap < W * total) return SZX_ENOSPC;
+    if (total && (!d_out || !aligned16(d_out))) return SZX_EINVAL;
+    DumpRes R;
+    if (!R.init(static_cast<cudaStream_t>(stream))) return SZX_ECUDA;
+    cudaStream_t s = R.s, s2 = R.s2;
+    uint64_t lmax = 16, wmax = 16;
+    for (auto& pt : parts) {
+        lmax = std::max(lmax, al16(pt.len));
+        wmax = std::max(wmax, szx_decompress_workspace_bytes(&pt.h));
+    }
+    void* buf[2] = {R.dalloc(lmax), R.dalloc(lmax)};
+    void* ws[2] = {R.dalloc(wmax), R.dalloc(wmax)};
+    int32_t* st = static_cast<int32_t*>(R.dalloc(4ull * parts.size()));
+    if (!buf[0] || !buf[1] || !ws[0] || !ws[1] || !st) return SZX_ENOMEM;
+    cudaMemsetAsync(st, 0, 4ull * parts.size(), s);
+    cudaEvent_t copied[2] = {R.event(), R.event()}, decoded[2] = {R.event(), R.event()};
+    uint8_t* out = static_cast<uint8_t*>(d_out);
+    for (size_t q = 0; q < parts.size(); q++) {
+        const Part& pt = parts[q];
+        if (q >= 2) cudaStreamWaitEvent(s2, decoded[q & 1], 0);  // the buffer's previous shard is decoded
+        if (cudaMemcpyAsync(buf[q & 1], hb + pt.off, pt.len, cudaMemcpyHostToDevice, s2) != cudaSuccess)
+            return SZX_ECUDA;
+        cudaEventRecord(copied[q & 1], s2);
+        cudaStreamWaitEvent(s, copied[q & 1], 0);
+        if (pt.h.n) {
+            int rc = szx_decompress_async(buf[q & 1], pt.len, &pt.h, out + W * pt.first, cap - W * pt.first, ws[q & 1],
+                                          wmax, st + q, s);
+            if (rc) return rc;
+        }
+        cudaEventRecord(decoded[q & 1], s);
+    }
+    std::vector<int32_t> hs(parts.size());
+    if (cudaMemcpyAsync(hs.data(), st, 4 * hs.size(), cudaMemcpyDeviceToHost, s) != cudaSuccess) return SZX_ECUDA;
+    if (cudaStreamSynchronize(s) != cudaSuccess) return SZX_ECUDA;
+    timing_resolve();
+    for (int32_t e : hs)
+        if (e) return e;
+    return (int64_t)total;
+}
+
 void szx_timing_enable(int on) {
     Timing& T = timing();
     std::lock_guard<std::mutex> g(T.mu);

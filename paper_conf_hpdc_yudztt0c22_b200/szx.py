@@ -67,6 +67,8 @@ def lib() -> ctypes.CDLL:
         "szx_decompress_quality_async": (i32, [vp, u64, ctypes.POINTER(_Header), vp, vp, u64, vp, u64, vp, vp,
                                                vp]),
         "szx_quality_finish": (None, [vp, vp]),
+        "szx_dump_host": (i64, [vp, i32, u64, i32, dbl, u32, u32, vp, u64, vp]),
+        "szx_load_host": (i64, [vp, u64, vp, u64, vp]),
         "szx_local_range": (i32, [vp, i32, u64, u32, vp, vp, u64, vp]),
         "szx_compress_shard_async": (i32, [vp, i32, u64, i32, dbl, vp, u32, vp, u64, vp, u64, vp, vp]),
         "szx_timing_enable": (None, [i32]),
@@ -89,7 +91,7 @@ EXPORTED = ["szx_compress_bound", "szx_compress_workspace_bytes", "szx_decompres
             "szx_compress", "szx_compress_ws", "szx_compress_async", "szx_read_header",
             "szx_decompress", "szx_decompress_blocks", "szx_decompress_ws", "szx_decompress_async", "szx_compress_host",
             "szx_decompress_host", "szx_decompress_quality", "szx_decompress_quality_async",
-            "szx_quality_finish", "szx_local_range", "szx_compress_shard_async",
+            "szx_quality_finish", "szx_dump_host", "szx_load_host", "szx_local_range", "szx_compress_shard_async",
             "szx_timing_enable", "szx_timing_reset", "szx_timing_read", "szx_launch_count",
             "szx_debug_set_r_bias", "szx_strerror"]
 
@@ -264,6 +266,48 @@ def decompress_quality(s: torch.Tensor, ref: torch.Tensor, out: torch.Tensor | N
                                      out.numel() * out.element_size(), q, _stream(stream))
     _check(r, "szx_decompress_quality")
     return out[:n], _quality_dict(list(q), n)
+
+
+def dump_host(x: torch.Tensor, eb: float, mode="rel", block_size: int = 128, parts: int = 8, out=None,
+              stream=None) -> torch.Tensor:
+    """Dump a CUDA tensor to host memory as an SZXC container of `parts` block-range shards,
+    compression of shard p+1 overlapping the copy-out of shard p (Fig. 16 analogue).  Returns a
+    uint8 CPU tensor view (pinned)."""
+    _require_cuda(x)
+    x = x.contiguous().view(-1)
+    dt = _dtype_code(x)
+    if out is None:
+        nb = (x.numel() + block_size - 1) // block_size
+        P = max(1, min(parts, max(nb, 1)))
+        per = (nb + P - 1) // P * block_size
+        out = torch.empty(32 + 32 * P + P * (compress_bound(per, dt, block_size) + 16), dtype=torch.uint8,
+                          pin_memory=True)
+    r = lib().szx_dump_host(x.data_ptr() if x.numel() else None, dt, x.numel(), _mode_code(mode), float(eb),
+                            block_size, parts, out.data_ptr(), out.numel(), _stream(stream))
+    _check(r, "szx_dump_host")
+    return out[:r]
+
+
+def load_host(s: torch.Tensor, out: torch.Tensor | None = None, device="cuda", stream=None) -> torch.Tensor:
+    """Load a host-resident stream or container (uint8 CPU tensor, ideally pinned) into a CUDA tensor,
+    the copy of shard q+1 overlapping the decode of shard q."""
+    if s.is_cuda:
+        raise ValueError("host tensor required")
+    head = s[:64].numpy().tobytes()
+    if head[:4] == b"SZXC":
+        n = struct.unpack_from("<Q", head, 16)[0]
+        off0 = struct.unpack_from("<Q", s[48:56].numpy().tobytes())[0]
+        dt = int(s[off0 + 5])
+    else:
+        h = read_header(head)
+        n, dt = h.n, h.dtype
+    tdt = torch.float32 if dt == F32 else torch.float64
+    if out is None:
+        out = torch.empty(max(n, 1), dtype=tdt, device=device)
+    r = lib().szx_load_host(s.data_ptr(), s.numel(), out.data_ptr(), out.numel() * out.element_size(),
+                            _stream(stream))
+    _check(r, "szx_load_host")
+    return out[:n]
 
 
 def compress_host(x, eb: float, mode="rel", block_size: int = 128, out=None, stream=None):
