@@ -130,10 +130,8 @@ __device__ inline DHdr read_dheader(const uint8_t* in, const DPlan& p) {
 
 __device__ inline void set_corrupt(int32_t* err) { atomicExch(err, -3); }
 
-// Exclusive scan of one value per thread over the group of NT threads
-// (named barrier 1, see group_sync); returns exclusive, sets *agg.
-template <int NT>
-__device__ inline uint64_t cta_scan(uint64_t v, uint64_t* agg, uint64_t* s_w /*[NT / 32]*/) {
+// 256-thread CTA exclusive scan of one value per thread; returns exclusive, sets *agg.
+__device__ inline uint64_t cta_scan256(uint64_t v, uint64_t* agg, uint64_t* s_w /*[8]*/) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     uint64_t incl = v;
 #pragma unroll
@@ -141,12 +139,12 @@ __device__ inline uint64_t cta_scan(uint64_t v, uint64_t* agg, uint64_t* s_w /*[
         uint64_t t = __shfl_up_sync(0xffffffffu, incl, o);
         if (lane >= o) incl += t;
     }
-    group_sync<NT>();  // s_w may still be read by a previous scan
+    __syncthreads();  // s_w may still be read by a previous scan
     if (lane == 31) s_w[warp] = incl;
-    group_sync<NT>();
+    __syncthreads();
     uint64_t wpre = 0, tot = 0;
 #pragma unroll
-    for (int i = 0; i < NT / 32; i++) {
+    for (int i = 0; i < 8; i++) {
         const uint64_t t = s_w[i];
         wpre += i < warp ? t : 0;
         tot += t;
@@ -179,17 +177,16 @@ __device__ inline uint64_t cta_scan(uint64_t v, uint64_t* agg, uint64_t* s_w /*[
 #ifndef SZX_PAIR
 #define SZX_PAIR 1   // float32 b = 128: two blocks per warp, a half-warp each
 #endif
-constexpr int kIndexChunkMax = 256;
+constexpr int kIndexChunk = 256;
 
 // Copy zs[i0, i0 + cnt) (cnt <= 32 * kIndexChunk) into shared memory with
 // aligned 16-byte loads.  The zsize section is 16-byte aligned and padded to
 // a multiple of 16 bytes, so the rounded-out loads stay inside it.
-template <int NT>
 __device__ inline void stage_u16(uint16_t* s_dst, const uint16_t* __restrict__ zs, uint64_t i0, uint64_t cnt) {
     const uint64_t a = i0 & ~uint64_t(7);
     const uint32_t head = (uint32_t)(i0 - a);
     const uint32_t nq = (uint32_t)((head + cnt + 7) / 8);
-    for (uint32_t q = threadIdx.x; q < nq; q += NT) {
+    for (uint32_t q = threadIdx.x; q < nq; q += kIndexChunk) {
         const uint4 v = *reinterpret_cast<const uint4*>(zs + a + 8 * q);
         const uint32_t e[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
@@ -200,10 +197,9 @@ __device__ inline void stage_u16(uint16_t* s_dst, const uint16_t* __restrict__ z
     }
 }
 
-template <int W, int NT>
+template <int W>
 __device__ inline void index_phase(const DPlan& p, const uint8_t* __restrict__ in, const DHdr& hd,
                                    uint16_t* s_zs, uint64_t* s_w) {
-    constexpr int kIndexChunk = NT;  // tiles per chunk: one per group thread
     const uint64_t G = gridDim.x, c = blockIdx.x;
     const uint64_t w0 = p.nWi * c / G, w1 = p.nWi * (c + 1) / G;
     const uint32_t* bm = reinterpret_cast<const uint32_t*>(in + kHeaderBytes);
@@ -226,8 +222,8 @@ __device__ inline void index_phase(const DPlan& p, const uint8_t* __restrict__ i
         const uint32_t x = word_at(w);
         cnt += __popc(x) | (nc_tile(w, x) << 32);
     }
-    const uint64_t aggP = cta_sum64<NT>(cnt, s_w);
-    const uint64_t exP = grid_excl_prefix<NT>(p.slot_a, p.res_a, &p.ctr[0], aggP, s_w);
+    const uint64_t aggP = cta_sum64(cnt, s_w);
+    const uint64_t exP = grid_excl_prefix(p.slot_a, p.res_a, &p.ctr[0], aggP, s_w);
     const uint64_t aggA = aggP & 0xFFFFFFFFu, exA = exP & 0xFFFFFFFFu;
     uint64_t runT = exP >> 32;
     const bool ok = exA + aggA <= hd.nnc;
@@ -237,15 +233,15 @@ __device__ inline void index_phase(const DPlan& p, const uint8_t* __restrict__ i
     uint64_t zsum = 0;
     if (ok) {
         if (one) {
-            stage_u16<NT>(s_zs, zs, exA, aggA);
-            group_sync<NT>();
+            stage_u16(s_zs, zs, exA, aggA);
+            __syncthreads();
             for (uint32_t j = threadIdx.x; j < aggA; j += kIndexChunk) zsum += s_zs[j];
         } else {
             for (uint64_t i = exA + threadIdx.x; i < exA + aggA; i += kIndexChunk) zsum += zs[i];
         }
     }
-    const uint64_t aggZ = cta_sum64<NT>(zsum, s_w);
-    const uint64_t exZ = grid_excl_prefix<NT>(p.slot_z, p.res_z, &p.ctr[3], aggZ, s_w);
+    const uint64_t aggZ = cta_sum64(zsum, s_w);
+    const uint64_t exZ = grid_excl_prefix(p.slot_z, p.res_z, &p.ctr[3], aggZ, s_w);
     // (3) per tile: ncpre and tbase
     uint64_t runA = exA, runZ = exZ;
     for (uint64_t wc = w0; wc < w1; wc += kIndexChunk) {
@@ -254,7 +250,7 @@ __device__ inline void index_phase(const DPlan& p, const uint8_t* __restrict__ i
         const uint32_t cw = __popc(word);
         const uint64_t isnc = w < w1 ? nc_tile(w, word) : 0u;
         uint64_t totP;
-        const uint64_t exq = cta_scan<NT>(cw | (isnc << 32), &totP, s_w);
+        const uint64_t exq = cta_scan256(cw | (isnc << 32), &totP, s_w);
         const uint64_t ex = exq & 0xFFFFFFFFu, tot = totP & 0xFFFFFFFFu;
         if (w < w1) {
             p.ncpre[w] = (uint32_t)(runA + ex);
@@ -262,18 +258,18 @@ __device__ inline void index_phase(const DPlan& p, const uint8_t* __restrict__ i
         }
         runT += totP >> 32;
         if (!one) {
-            if (ok) stage_u16<NT>(s_zs, zs, runA, tot);
-            group_sync<NT>();
+            if (ok) stage_u16(s_zs, zs, runA, tot);
+            __syncthreads();
         }
         uint64_t sum = 0;
         if (ok)
             for (uint32_t j = 0; j < cw; j++) sum += s_zs[ex + j];
         uint64_t totz;
-        const uint64_t exz = cta_scan<NT>(sum, &totz, s_w);
+        const uint64_t exz = cta_scan256(sum, &totz, s_w);
         if (w < w1) p.tbase[w] = runZ + exz;
         runA += tot;
         runZ += totz;
-        group_sync<NT>();  // s_zs is refilled by the next chunk
+        __syncthreads();  // s_zs is refilled by the next chunk
     }
     if (threadIdx.x == 0) {
         if (!ok) set_corrupt(p.err);
@@ -680,7 +676,7 @@ struct DecWCfg {
 #endif
     static constexpr int FILLW = SZX_FILLW;         // fill warps per CTA (the rest decode)
     static constexpr int SMEM = NWARP * 2 * SLOT_ALLOC;
-    static_assert(SMEM >= kIndexChunkMax * 32 * 2, "index-phase scratch aliases the slots");
+    static_assert(SMEM >= kIndexChunk * 32 * 2, "index-phase scratch aliases the slots");
 };
 
 // Per-tile metadata a warp needs before it can store anything.
@@ -717,16 +713,10 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
     }
     // index phase (the shared staging slots double as its scratch), then a
     // grid barrier: tiles are decoded by whichever warp grabs them
-    // grid barrier; run by the decode warps [0, NIDX) only: the fill warps (the
-    // last FILLW) need nothing but the bitmap and the mu array, so they start
-    // streaming the constant blocks at once and wait for the barrier only
-    // before they help with the nonconstant tiles
-    constexpr int NIDX = (C::NWARP - C::FILLW) * 32;
-    const bool fill_warp = (int)(threadIdx.x >> 5) >= C::NWARP - C::FILLW;
-    if (!fill_warp) {
-        index_phase<W, NIDX>(p, in, hd, reinterpret_cast<uint16_t*>(dsm), s_w);
-        grid_barrier<NIDX>(&p.ctr[2]);
-    }
+    index_phase<W>(p, in, hd, reinterpret_cast<uint16_t*>(dsm), s_w);
+    if (SZX_EXP & 32) return;
+    grid_barrier(&p.ctr[2]);
+    if (SZX_EXP & 16) return;
     const int lane = threadIdx.x & 31;
     const uint32_t* bm = reinterpret_cast<const uint32_t*>(in + kHeaderBytes);
     const uint16_t* zs = reinterpret_cast<const uint16_t*>(in + hd.off_zs);
@@ -791,7 +781,7 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
             mul = mn;
         }
     };
-    uint32_t n_nct = 0;  // read once the index phase is complete (grid barrier)
+    const uint32_t n_nct = *p.n_nctile;
 
     auto load_meta = [&](uint64_t t, TileMeta<U>& m) {
         uint32_t word = bm[t];
@@ -1023,15 +1013,16 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
     };
     // Each warp drains its own queue first, then helps with the other one, so
     // the split adapts to the field's fraction of nonconstant blocks.
-    if (fill_warp) {
+    if (SZX_EXP & 256) {
+        if ((int)(threadIdx.x >> 5) < C::FILLW) fill_loop();
+        return;
+    }
+    if ((int)(threadIdx.x >> 5) < C::FILLW) {
         fill_loop();
-        grid_wait(&p.ctr[2]);
-        n_nct = *p.n_nctile;
-        nc_loop();
+        if (SZX_SWITCH & 2) nc_loop();
     } else {
-        n_nct = *p.n_nctile;
         nc_loop();
-        fill_loop();
+        if (SZX_SWITCH & 1) fill_loop();
     }
     if constexpr (QUAL) qa.flush(p.qual);
 }

@@ -301,26 +301,14 @@ __device__ inline uint32_t ld_acquire_u32(const uint32_t* p) {
     return v;
 }
 
-// The helpers below synchronise a GROUP of the CTA's threads: threads
-// [0, NT) with named barrier 1 (the decoder's index warps, while its fill
-// warps already stream), or the whole CTA when NT == 0.
-template <int NT>
-__device__ __forceinline__ void group_sync() {
-    if constexpr (NT == 0) __syncthreads();
-    else asm volatile("bar.sync 1, %0;" ::"n"(NT) : "memory");
-}
-template <int NT>
-__device__ __forceinline__ int group_size() { return NT ? NT : (int)blockDim.x; }
-
-// Sum over the group (a multiple of 32 threads, <= 1024); result in every
-// thread.  s_w: shared scratch of 32 u64.
-template <int NT = 0>
+// Sum over the CTA (any blockDim that is a multiple of 32, <= 1024); result
+// in every thread.  s_w: shared scratch of 32 u64.
 __device__ inline uint64_t cta_sum64(uint64_t v, uint64_t* s_w) {
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarp = group_size<NT>() >> 5;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarp = blockDim.x >> 5;
     v = warp_sum64(v);
-    group_sync<NT>();  // s_w may still be read by a previous call
+    __syncthreads();  // s_w may still be read by a previous call
     if (lane == 0) s_w[warp] = v;
-    group_sync<NT>();
+    __syncthreads();
     uint64_t t = 0;
     for (int i = 0; i < nwarp; i++) t += s_w[i];
     return t;
@@ -333,36 +321,34 @@ __device__ inline uint64_t cta_sum64(uint64_t v, uint64_t* s_w) {
 // about three round trips, with no chained look-back and no all-to-all
 // polling.  `res` [gridDim.x] and `*arrive` must be zero.
 constexpr uint64_t kSlotFlag = 1ull << 63;
-template <int NT = 0>
 __device__ inline uint64_t grid_excl_prefix(uint64_t* slots, uint64_t* res, uint32_t* arrive, uint64_t agg,
                                             uint64_t* s_w /*[32]*/) {
     __shared__ uint32_t s_last;
     __shared__ uint64_t s_val;
     const uint32_t G = gridDim.x;
-    const int nth = group_size<NT>();
     if (threadIdx.x == 0) {
         st_relaxed(&slots[blockIdx.x], agg);
         __threadfence();
         s_last = atomicAdd(arrive, 1u) == G - 1;
     }
-    group_sync<NT>();
+    __syncthreads();
     if (s_last) {
         __threadfence();
         uint64_t run = 0;
-        for (uint32_t b0 = 0; b0 < G; b0 += nth) {
+        for (uint32_t b0 = 0; b0 < G; b0 += blockDim.x) {
             const uint32_t i = b0 + threadIdx.x;
             const uint64_t v = i < G ? ld_relaxed(&slots[i]) : 0;
-            // group exclusive scan of v
-            const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarp = nth >> 5;
+            // CTA exclusive scan of v
+            const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarp = blockDim.x >> 5;
             uint64_t incl = v;
 #pragma unroll
             for (int o = 1; o < 32; o <<= 1) {
                 const uint64_t t = __shfl_up_sync(0xffffffffu, incl, o);
                 if (lane >= o) incl += t;
             }
-            group_sync<NT>();
+            __syncthreads();
             if (lane == 31) s_w[warp] = incl;
-            group_sync<NT>();
+            __syncthreads();
             uint64_t wpre = 0, tot = 0;
             for (int k = 0; k < nwarp; k++) {
                 wpre += k < warp ? s_w[k] : 0;
@@ -377,32 +363,21 @@ __device__ inline uint64_t grid_excl_prefix(uint64_t* slots, uint64_t* res, uint
         while (!((v = ld_relaxed(&res[blockIdx.x])) & kSlotFlag)) __nanosleep(32);
         s_val = v & ~kSlotFlag;
     }
-    group_sync<NT>();
+    __syncthreads();
     return s_val;
 }
 
-// Grid barrier over the groups of every CTA: every global write made by any
-// group thread of any CTA before the call is visible to every group thread
-// after it.  `ctr` must be zero.  Threads outside the group that need the
-// same guarantee call grid_wait(ctr).
-template <int NT = 0>
+// Grid barrier: every global write made by any thread of any CTA before the
+// call is visible to every thread after it.  `ctr` must be zero.
 __device__ inline void grid_barrier(uint32_t* ctr) {
-    group_sync<NT>();
+    __syncthreads();
     if (threadIdx.x == 0) {
         __threadfence();
         atomicAdd(ctr, 1u);
         while (ld_acquire_u32(ctr) < gridDim.x) __nanosleep(64);
         __threadfence();
     }
-    group_sync<NT>();
-}
-// One warp waits until every CTA has passed grid_barrier(ctr).
-__device__ inline void grid_wait(const uint32_t* ctr) {
-    if ((threadIdx.x & 31) == 0) {
-        while (ld_acquire_u32(ctr) < gridDim.x) __nanosleep(64);
-        __threadfence();
-    }
-    __syncwarp();
+    __syncthreads();
 }
 
 }  // namespace szx
