@@ -27,8 +27,10 @@
  *     corrupt stream is reported as SZX_ECORRUPT without out-of-bounds
  *     accesses.  There is no CPU fallback: without a CUDA device every
  *     compute call returns SZX_ECUDA.
- *   - Supported GPU block sizes b: 128 and 256 (b = 128 is the paper's
- *     choice).  Max elements per stream: 2^36.
+ *   - Supported GPU block sizes b: 32, 64, 128 and 256 (a warp per block,
+ *     b / 32 values per lane; b = 128 is the paper's choice, P:L2099-2105,
+ *     and the one the fast paths target; the block-size study is Sec. 5.3,
+ *     P:L1748-2188).  Max elements per stream: 2^36.
  */
 #ifndef SZX_B200_H
 #define SZX_B200_H

@@ -139,7 +139,7 @@ uint64_t* pinned_u64() {
 
 bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; }
 int wbytes(szx_dtype_t dt) { return dt == SZX_F64 ? 8 : 4; }
-bool block_ok(uint32_t b) { return b == 128 || b == 256; }
+bool block_ok(uint32_t b) { return b == 32 || b == 64 || b == 128 || b == 256; }
 uint64_t cdiv(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
 
 // ------------------------------------------------------------ compress layout
@@ -210,11 +210,18 @@ void carve(K k) {
     if (SZX_CARVE) cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, SZX_CARVE);
 }
 
+// blocks per warp in flight in the stats pass: 128 bytes of loads per lane (at most 16 blocks)
+template <typename T, int VPL>
+constexpr int stats_unroll() {
+    constexpr int u = 128 / (VPL * (int)sizeof(T));
+    return u < 1 ? 1 : (u > 16 ? 16 : u);
+}
+
 template <typename T, int VPL>
 void set_smem_attrs() {
     static bool done = false;
     if (done) return;
-    constexpr int UNR = 128 / (VPL * (int)sizeof(T)) > 0 ? 128 / (VPL * (int)sizeof(T)) : 1;
+    constexpr int UNR = stats_unroll<T, VPL>();
     carve(k_block_stats<T, VPL, UNR>);
     carve(k_classify<T>);
     carve(k_enc_size<T, VPL>);
@@ -233,7 +240,7 @@ void set_smem_attrs() {
 template <typename T, int VPL>
 void enqueue_stats(const void* d_in, const Plan& p, int want_range, cudaStream_t s) {
     set_smem_attrs<T, VPL>();
-    constexpr int UNR = 128 / (VPL * (int)sizeof(T)) > 0 ? 128 / (VPL * (int)sizeof(T)) : 1;
+    constexpr int UNR = stats_unroll<T, VPL>();
     static int occ = 0;
     if (!occ) {
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_block_stats<T, VPL, UNR>, 256, 0);
@@ -314,11 +321,17 @@ int enqueue_compress(const void* d_in, szx_dtype_t dt, uint64_t n, szx_ebmode_t 
 template <int V> struct IC { static constexpr int value = V; };
 template <typename F>
 void dispatch(szx_dtype_t dt, uint32_t b, F&& f) {
-    if (dt == SZX_F32) {
-        if (b == 128) f(float(), IC<4>()); else f(float(), IC<8>());
-    } else {
-        if (b == 128) f(double(), IC<4>()); else f(double(), IC<8>());
-    }
+    // b = 32 x VPL: a warp owns a block, VPL values per lane
+    auto go = [&](auto tag) {
+        switch (b) {
+            case 32: f(tag, IC<1>()); break;
+            case 64: f(tag, IC<2>()); break;
+            case 128: f(tag, IC<4>()); break;
+            default: f(tag, IC<8>()); break;
+        }
+    };
+    if (dt == SZX_F32) go(float());
+    else go(double());
 }
 
 int64_t finish_sync(cudaStream_t s, const uint64_t* d_val, uint64_t* out_val) {

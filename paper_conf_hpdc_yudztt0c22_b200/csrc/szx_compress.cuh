@@ -64,10 +64,11 @@ __device__ inline int load_lane(const T* __restrict__ x, uint64_t n, uint64_t k,
     constexpr int B = 32 * VPL;
     const uint64_t first = k * B + (uint64_t)lane * VPL;
     if ((k + 1) * B <= n) {
-        constexpr int NV = VPL * (int)sizeof(T) / 16;
-        const uint4* p = reinterpret_cast<const uint4*>(x + first);
+        using LY = Lay<T, VPL>;
+        using V = typename LY::V;
+        const V* p = reinterpret_cast<const V*>(x + first);
 #pragma unroll
-        for (int q = 0; q < NV; q++) reinterpret_cast<uint4*>(v)[q] = ld_stream16(p + q);
+        for (int q = 0; q < LY::NQ; q++) reinterpret_cast<V*>(v)[q] = ld_stream<V>(p + q);
         return VPL;
     }
     int cnt = first >= n ? 0 : (int)umin64(VPL, n - first);
@@ -128,17 +129,19 @@ __global__ void __launch_bounds__(256) k_block_stats(const T* __restrict__ x, Pl
         }
     };
     constexpr int B = 32 * VPL;
-    constexpr int NV = VPL * (int)sizeof(T) / 16;   // 16-byte loads per lane per block
+    using LY = Lay<T, VPL>;
+    using V = typename LY::V;
+    constexpr int NV = LY::NQ;                       // chunk loads per lane per block
     const uint64_t nBf = p.n / B;                    // full blocks
     uint64_t k0 = gw * UNR;
     // fast path: UNR full blocks per warp, all loads issued first, no bounds checks
     for (; k0 + UNR <= nBf; k0 += nw * UNR) {
-        const uint4* src = reinterpret_cast<const uint4*>(x + k0 * B) + lane * NV;
+        const V* src = reinterpret_cast<const V*>(x + k0 * B) + lane * NV;
         T v[UNR][VPL];
 #pragma unroll
         for (int u = 0; u < UNR; u++)
 #pragma unroll
-            for (int q = 0; q < NV; q++) reinterpret_cast<uint4*>(v[u])[q] = ld_stream16(src + u * (B / 4 * sizeof(T) / 4) + q);
+            for (int q = 0; q < NV; q++) reinterpret_cast<V*>(v[u])[q] = ld_stream<V>(src + u * (B * (int)sizeof(T) / LY::CB) + q);
 #pragma unroll
         for (int u = 0; u < UNR; u++) block(v[u], VPL, k0 + u);
     }
@@ -488,10 +491,14 @@ __device__ inline void pack_red(const typename Traits<T>::U (&u)[VPL], const Lan
     const int s = raw ? 0 : ((8 - (lc.R & 7)) & 7);
     const int req = (lc.R + s) >> 3;
     if (lane == 0) red_or_byte(dst, (uint32_t)lc.R);
+    if constexpr (VPL >= 4) {
 #pragma unroll
-    for (int q = 0; q < VPL / 4; q++) {
-        const int cb = lane * (VPL / 4) + q;
-        if (cb < ncode) red_or_byte(dst + 1 + cb, lc.leads >> (8 * q));
+        for (int q = 0; q < VPL / 4; q++) {
+            const int cb = lane * (VPL / 4) + q;
+            if (cb < ncode) red_or_byte(dst + 1 + cb, lc.leads >> (8 * q));
+        }
+    } else {  // 4 / VPL lanes share a code byte
+        if ((int)code_byte<VPL>(lane) < ncode) red_or_byte(dst + 1 + code_byte<VPL>(lane), lc.leads << code_shift<VPL>(lane));
     }
     uint32_t a = dst + 1 + ncode + lc.mexcl;
 #pragma unroll
@@ -756,7 +763,8 @@ struct SizeCfg {
     static constexpr int W = Traits<T>::W;
     static constexpr int B = 32 * VPL;
     static constexpr int BW = B * W;
-    static constexpr int QV = VPL * W / 16;      // 16-byte chunks per lane per block
+    static constexpr int QV = Lay<T, VPL>::NQ;   // chunks per lane per block
+    static constexpr int CB = Lay<T, VPL>::CB;   // chunk bytes
     static constexpr int NB = 4;                 // blocks per batch
     static constexpr int WARP_BYTES = 2 * NB * BW;
     static constexpr int SMEM = 8 * WARP_BYTES;
@@ -897,7 +905,7 @@ __global__ void __launch_bounds__(256) k_enc_size(const T* __restrict__ x, Plan 
                     const T* src = x + (uint64_t)k * B + lane * VPL;
 #pragma unroll
                     for (int q = 0; q < C::QV; q++)
-                        cp_async16(st + j * C::BW + (lane * C::QV + q) * 16, src + q * (16 / W));
+                        cp_async_chunk<C::CB>(st + j * C::BW + (lane * C::QV + q) * C::CB, src + q * (C::CB / W));
                 }
             }
             cp_async_commit();
@@ -929,8 +937,9 @@ __global__ void __launch_bounds__(256) k_enc_size(const T* __restrict__ x, Plan 
                     T x0[VPL], x1[VPL];
 #pragma unroll
                     for (int q = 0; q < C::QV; q++) {
-                        reinterpret_cast<uint4*>(x0)[q] = lds_u128(st + j * C::BW + (lane * C::QV + q) * 16);
-                        reinterpret_cast<uint4*>(x1)[q] = lds_u128(st + (j + 1) * C::BW + (lane * C::QV + q) * 16);
+                        using V = typename Lay<T, VPL>::V;
+                        reinterpret_cast<V*>(x0)[q] = lds_chunk<V>(st + j * C::BW + (lane * C::QV + q) * C::CB);
+                        reinterpret_cast<V*>(x1)[q] = lds_chunk<V>(st + (j + 1) * C::BW + (lane * C::QV + q) * C::CB);
                     }
                     int R0 = (int)(rec0 & 0x7F), R1 = (int)(rec1 & 0x7F);
                     uint32_t z0, z1 = 0u;
@@ -967,8 +976,10 @@ __global__ void __launch_bounds__(256) k_enc_size(const T* __restrict__ x, Plan 
                     LaneCode lc;
                     if (k < nBfull) {
 #pragma unroll
-                        for (int q = 0; q < C::QV; q++)
-                            reinterpret_cast<uint4*>(xv)[q] = lds_u128(st + (j + h) * C::BW + (lane * C::QV + q) * 16);
+                        for (int q = 0; q < C::QV; q++) {
+                            using V = typename Lay<T, VPL>::V;
+                            reinterpret_cast<V*>(xv)[q] = lds_chunk<V>(st + (j + h) * C::BW + (lane * C::QV + q) * C::CB);
+                        }
                         encode_block<T, VPL>(xv, VPL, B, mu, (int)(rec & 0x7F), (rec & 0x80) != 0, eb, uu, lc);
                     } else {
                         const int cnt = load_lane<T, VPL>(x, p.n, k, lane, xv);
@@ -1095,7 +1106,8 @@ struct WriteCfg {
     static constexpr int W = Traits<T>::W;
     static constexpr int B = 32 * VPL;
     static constexpr int BW = B * W;
-    static constexpr int QV = VPL * W / 16;
+    static constexpr int QV = Lay<T, VPL>::NQ;
+    static constexpr int CB = Lay<T, VPL>::CB;
     static constexpr int TB = kWriteTile;
     static constexpr int NWARP = 8;
     static constexpr int BPW = TB / NWARP;
@@ -1137,7 +1149,7 @@ __global__ void __launch_bounds__(256) k_enc_write(const T* __restrict__ x, Plan
         if (tfull || (ncw + j < nnc && k < nBfull)) {
             const T* src = x + (uint64_t)k * C::B + lane * VPL;
 #pragma unroll
-            for (int q = 0; q < C::QV; q++) cp_async16(sin + j * C::BW + (lane * C::QV + q) * 16, src + q * (16 / W));
+            for (int q = 0; q < C::QV; q++) cp_async_chunk<C::CB>(sin + j * C::BW + (lane * C::QV + q) * C::CB, src + q * (C::CB / W));
         }
     }
     cp_async_commit();
@@ -1205,8 +1217,10 @@ __global__ void __launch_bounds__(256) k_enc_write(const T* __restrict__ x, Plan
         LaneCode lc;
         if (k < nBfull) {
 #pragma unroll
-            for (int q = 0; q < C::QV; q++)
-                reinterpret_cast<uint4*>(xv)[q] = lds_u128(sin + j * C::BW + (lane * C::QV + q) * 16);
+            for (int q = 0; q < C::QV; q++) {
+                using V = typename Lay<T, VPL>::V;
+                reinterpret_cast<V*>(xv)[q] = lds_chunk<V>(sin + j * C::BW + (lane * C::QV + q) * C::CB);
+            }
             if constexpr (sizeof(T) == 4 && VPL == 4) {
                 Lane4 e;
                 lane_encode_f32x4(xv, cmu, R, e);

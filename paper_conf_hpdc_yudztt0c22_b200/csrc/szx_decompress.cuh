@@ -74,15 +74,15 @@ struct QualAcc {
         kmx = fin && k > kmx ? k : kmx;
     }
     // 16-byte chunks of decoded values against the same chunks of the original
-    template <typename T, int NV>
-    __device__ __forceinline__ void add16(const uint4* ref, const uint4 (&v)[NV]) {
+    template <typename T, int NV, typename V = uint4>
+    __device__ __forceinline__ void add16(const V* ref, const V (&v)[NV]) {
 #pragma unroll
         for (int q = 0; q < NV; q++) {
-            const uint4 r = ld_stream16(ref + q);
+            const V r = ld_stream<V>(ref + q);
             const T* a = reinterpret_cast<const T*>(&r);
             const T* b = reinterpret_cast<const T*>(&v[q]);
 #pragma unroll
-            for (int i = 0; i < 16 / (int)sizeof(T); i++) add<T>(a[i], b[i]);
+            for (int i = 0; i < (int)sizeof(V) / (int)sizeof(T); i++) add<T>(a[i], b[i]);
         }
     }
     // warp reduction, then one set of atomics per warp
@@ -289,10 +289,11 @@ __device__ inline void store_lane(T* __restrict__ y, uint64_t n, uint64_t k, int
     constexpr int B = 32 * VPL;
     const uint64_t first = k * B + (uint64_t)lane * VPL;
     if ((k + 1) * B <= n) {
-        constexpr int NV = VPL * (int)sizeof(T) / 16;
-        uint4* q = reinterpret_cast<uint4*>(y + first);
+        using LY = Lay<T, VPL>;
+        using V = typename LY::V;
+        V* q = reinterpret_cast<V*>(y + first);
 #pragma unroll
-        for (int i = 0; i < NV; i++) q[i] = reinterpret_cast<const uint4*>(v)[i];
+        for (int i = 0; i < LY::NQ; i++) q[i] = reinterpret_cast<const V*>(v)[i];
         return;
     }
 #pragma unroll
@@ -358,10 +359,15 @@ __device__ inline bool decode_block_g(const Src src, uint32_t z, int len, T mu,
     const int cnt = first >= len ? 0 : min(VPL, len - first);
     // (1) read the leading numbers
     uint32_t leads = 0;
+    if constexpr (VPL >= 4) {
 #pragma unroll
-    for (int q = 0; q < VPL / 4; q++) {
-        const int cb = lane * (VPL / 4) + q;
-        if (cb < ncode) leads |= src.u8(1 + cb) << (8 * q);
+        for (int q = 0; q < VPL / 4; q++) {
+            const int cb = lane * (VPL / 4) + q;
+            if (cb < ncode) leads |= src.u8(1 + cb) << (8 * q);
+        }
+    } else {  // 4 / VPL lanes share a code byte
+        if ((int)code_byte<VPL>(lane) < ncode)
+            leads = (src.u8(1 + code_byte<VPL>(lane)) >> code_shift<VPL>(lane)) & ((1u << (2 * VPL)) - 1u);
     }
     uint32_t m = 0;
 #pragma unroll
@@ -598,6 +604,7 @@ __device__ inline bool decode_full_g(const Src src, uint32_t z, T mu, T (&out)[V
     uint32_t leads = 0;
 #pragma unroll
     for (int q = 0; q < VPL / 4; q++) leads |= src.u8(1 + lane * (VPL / 4) + q) << (8 * q);
+    if constexpr (VPL < 4) leads = (src.u8(1 + code_byte<VPL>(lane)) >> code_shift<VPL>(lane)) & ((1u << (2 * VPL)) - 1u);
     uint32_t m = 0;
 #pragma unroll
     for (int i = 0; i < VPL; i++) {
@@ -648,6 +655,15 @@ __device__ inline bool decode_full_g(const Src src, uint32_t z, T mu, T (&out)[V
     return true;
 }
 
+// store of decompressed output (streaming: evict-first)
+template <typename V>
+__device__ inline void st_out(V* p, V v) {
+#if SZX_STCS
+    __stcs(p, v);
+#else
+    *p = v;
+#endif
+}
 // 16-byte store of decompressed output
 __device__ inline void st_out16(uint4* p, uint4 v) {
 #if SZX_STCS
@@ -698,8 +714,10 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
     constexpr int B = 32 * VPL;
     constexpr int TB = kTileBlocks;
     constexpr int MAXZ = 1 + B / 4 + W * B;
-    constexpr int NV = VPL * W / 16;  // 16-byte stores per lane per block
-    constexpr int QB = B * W / 16;    // 16-byte chunks per block
+    using LY = Lay<T, VPL>;
+    using V = typename LY::V;
+    constexpr int NV = LY::NQ;        // chunk stores per lane per block
+    constexpr int QB = B * W / LY::CB;  // chunks per block
     extern __shared__ __align__(16) uint8_t dsm[];
     __shared__ uint64_t s_w[32];
     QualAcc qa;
@@ -762,7 +780,7 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
             uint32_t wn = 0;
             U mn = 0;
             if (tn < fill_end) { wn = bm[tn]; mn = mus[tn * TB + lane]; }
-            uint4* yq = reinterpret_cast<uint4*>(y + t * TB * B + lane * VPL);
+            V* yq = reinterpret_cast<V*>(y + t * TB * B + lane * VPL);
 #pragma unroll 2
             for (uint32_t m = ~word & rmask(t); m; m &= m - 1) {
                 const int j = __ffs(m) - 1;
@@ -771,10 +789,10 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
 #pragma unroll
                 for (int q = 0; q < VPL; q++) v[q] = TR::from(mb);
 #pragma unroll
-                for (int q = 0; q < NV; q++) st_out16(yq + j * QB + q, reinterpret_cast<const uint4*>(v)[q]);
+                for (int q = 0; q < NV; q++) st_out(yq + j * QB + q, reinterpret_cast<const V*>(v)[q]);
                 if constexpr (QUAL)
-                    qa.add16<T, NV>(reinterpret_cast<const uint4*>(ref + t * TB * B + lane * VPL) + j * QB,
-                                    reinterpret_cast<const uint4(&)[NV]>(v));
+                    qa.add16<T, NV, V>(reinterpret_cast<const V*>(ref + t * TB * B + lane * VPL) + j * QB,
+                                       reinterpret_cast<const V(&)[NV]>(v));
             }
             t = tn;
             word = wn;
@@ -860,7 +878,7 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
     auto decode_seg = [&](uint64_t t, const TileMeta<U>& m, const TileZ& z, const SegT& sg, int sl) {
         const uint32_t sbase = slot0 + sl * C::SLOT_ALLOC +
                                (uint32_t)(reinterpret_cast<uintptr_t>(pl + m.base + sg.off0) & 15) - sg.off0;
-        uint4* yq = reinterpret_cast<uint4*>(y + t * TB * B + lane * VPL);
+        V* yq = reinterpret_cast<V*>(y + t * TB * B + lane * VPL);
         const uint32_t rm = rmask(t);
         // blocks whose rank lies in [r0, r1), restricted to the requested range;
         // lane j holds block j's payload offset and size (one shuffle each per segment)
@@ -917,10 +935,10 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
                 continue;
             }
 #pragma unroll
-            for (int q = 0; q < NV; q++) st_out16(yq + j * QB + q, reinterpret_cast<const uint4*>(v)[q]);
+            for (int q = 0; q < NV; q++) st_out(yq + j * QB + q, reinterpret_cast<const V*>(v)[q]);
             if constexpr (QUAL)
-                qa.add16<T, NV>(reinterpret_cast<const uint4*>(ref + t * TB * B + lane * VPL) + j * QB,
-                                reinterpret_cast<const uint4(&)[NV]>(v));
+                qa.add16<T, NV, V>(reinterpret_cast<const V*>(ref + t * TB * B + lane * VPL) + j * QB,
+                                   reinterpret_cast<const V(&)[NV]>(v));
         }
     };
     // the partial last tile: generic decoder, straight from global memory

@@ -256,6 +256,64 @@ __device__ inline uint4 ld_stream16(const void* p) {
     return v;
 }
 
+// ---------------------------------------------------------------- lane chunks
+// A lane's VPL values of a block are LB = VPL x W contiguous bytes, moved as
+// NQ chunks of CB = min(LB, 16) bytes (16-byte vectors for b >= 128 float32,
+// 4- or 8-byte words for the small blocks b = 32 / 64).
+template <int CB> struct ChunkT;
+template <> struct ChunkT<4> { using V = uint32_t; };
+template <> struct ChunkT<8> { using V = uint2; };
+template <> struct ChunkT<16> { using V = uint4; };
+template <typename T, int VPL>
+struct Lay {
+    static constexpr int LB = VPL * (int)sizeof(T);
+    static constexpr int CB = LB < 16 ? LB : 16;
+    static constexpr int NQ = LB / CB;
+    using V = typename ChunkT<CB>::V;
+};
+// streaming load of one chunk (read once; do not keep in L1)
+template <typename V>
+__device__ inline V ld_stream(const V* p);
+template <>
+__device__ inline uint4 ld_stream<uint4>(const uint4* p) { return ld_stream16(p); }
+template <>
+__device__ inline uint2 ld_stream<uint2>(const uint2* p) {
+    uint2 v;
+    asm volatile("ld.global.nc.L1::no_allocate.v2.u32 {%0,%1}, [%2];" : "=r"(v.x), "=r"(v.y) : "l"(p));
+    return v;
+}
+template <>
+__device__ inline uint32_t ld_stream<uint32_t>(const uint32_t* p) {
+    uint32_t v;
+    asm volatile("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(v) : "l"(p));
+    return v;
+}
+// shared-memory load of one chunk
+template <typename V>
+__device__ inline V lds_chunk(uint32_t a);
+template <>
+__device__ inline uint4 lds_chunk<uint4>(uint32_t a) { return lds_u128(a); }
+template <>
+__device__ inline uint2 lds_chunk<uint2>(uint32_t a) {
+    uint2 v;
+    asm volatile("ld.shared.v2.u32 {%0,%1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(a));
+    return v;
+}
+template <>
+__device__ inline uint32_t lds_chunk<uint32_t>(uint32_t a) { return lds_u32(a); }
+// asynchronous global -> shared copy of one chunk
+template <int CB>
+__device__ inline void cp_async_chunk(uint32_t saddr, const void* g) {
+    if constexpr (CB == 16) cp_async16(saddr, g);
+    else asm volatile("cp.async.ca.shared.global [%0], [%1], %2;" ::"r"(saddr), "l"(g), "n"(CB) : "memory");
+}
+// Lead codes of a lane (2 bits per value, LSB-first, reading R8): byte
+// lane*VPL/4 of the code array, at bit (2*VPL*lane) % 8 when VPL < 4.
+template <int VPL>
+__device__ inline uint32_t code_byte(int lane) { return (uint32_t)(lane * VPL / 4); }
+template <int VPL>
+__device__ inline uint32_t code_shift(int lane) { return VPL >= 4 ? 0u : (uint32_t)((2 * VPL * lane) & 7); }
+
 // ---------------------------------------------------------------- addresses
 __device__ inline uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 

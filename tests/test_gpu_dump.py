@@ -50,9 +50,12 @@ def test_dump_load_nyx_and_streams():
     y = szx.load_host(c)
     assert torch.equal(y, szx.decompress(torch.from_numpy(ref).cuda()))
     # a bare SZX1 stream loads too, and 256-blocks
-    s = oracle.compress(x.numpy(), 1e-3, oracle.REL, 256)
-    y2 = szx.load_host(torch.from_numpy(s).pin_memory())
-    assert np.array_equal(y2.cpu().numpy().view(np.uint32), oracle.decompress(s).view(np.uint32))
+    for b in (32, 64, 256):
+        s = oracle.compress(x.numpy(), 1e-3, oracle.REL, b)
+        y2 = szx.load_host(torch.from_numpy(s).pin_memory())
+        assert np.array_equal(y2.cpu().numpy().view(np.uint32), oracle.decompress(s).view(np.uint32))
+        c = szx.dump_host(xd, 1e-3, "rel", b, 5)
+        assert c.numpy().tobytes() == oracle.container_compress(x.numpy(), 1e-3, oracle.REL, b, 5).tobytes()
 
 
 def test_load_rejects_corrupt_and_dump_checks_capacity():

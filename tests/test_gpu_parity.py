@@ -75,7 +75,7 @@ SMALL = {
 def test_parity_small_fields(name, dt):
     x = SMALL[name]().astype(dt)
     for mode, eb in (("rel", 1e-2), ("rel", 1e-3), ("rel", 1e-4), ("abs", 1e-3)):
-        for b in (128, 256):
+        for b in (32, 64, 128, 256):
             _parity(x, eb, mode, b, f"{name}/{dt.__name__}/{mode}{eb}/b{b}")
 
 
@@ -84,7 +84,7 @@ def test_parity_small_fields(name, dt):
 def test_parity_sizes_and_tails(n):
     x = synth.random_mix(max(n, 1), 100 + n).numpy()[:n]
     for dt in (np.float32, np.float64):
-        for b in (128, 256):
+        for b in (32, 64, 128, 256):
             _parity(x.astype(dt), 1e-3, "rel", b, f"n={n}/{dt.__name__}/b{b}")
 
 

@@ -65,7 +65,7 @@ FIELDS = {
 def test_quality_matches_oracle(name, dt):
     x = FIELDS[name]().astype(dt)
     for mode, eb in (("rel", 1e-3), ("abs", 1e-2)):
-        for b in (128, 256):
+        for b in (32, 64, 128, 256):
             _check(x, eb, mode, b, f"{name}/{dt.__name__}/{mode}{eb}/b{b}")
 
 
