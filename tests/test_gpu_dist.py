@@ -71,6 +71,14 @@ def test_sharded_container_matches_oracle(P, dt, mode):
     assert np.array_equal(y.view(ui), oracle.decompress(ref).view(ui))
 
 
+@pytest.mark.parametrize("b", [32, 64, 256])
+def test_sharded_container_small_and_large_blocks(b):
+    x = synth.random_mix(300_007, 41).numpy()
+    c = _compress_sharded(torch.from_numpy(x).cuda(), 5, 1e-3, "rel", b).cpu().numpy()
+    ref = oracle.container_compress(x, 1e-3, oracle.REL, b, 5)
+    assert c.tobytes() == ref.tobytes()
+
+
 def test_sharded_special_values_and_empty_shards():
     x = synth.special_values(1000, 3).numpy()  # 8 blocks, 16 shards -> empty shards
     c = _compress_sharded(torch.from_numpy(x).cuda(), 16, 1e-2, "rel", 128).cpu().numpy()
@@ -100,7 +108,7 @@ def _blocks_ref(yref: np.ndarray, b: int, k0: int, nb: int) -> np.ndarray:
 
 
 @pytest.mark.parametrize("dt", [np.float32, np.float64])
-@pytest.mark.parametrize("b", [128, 256])
+@pytest.mark.parametrize("b", [32, 64, 128, 256])
 def test_decompress_blocks_matches_oracle_slices(dt, b):
     """1 stream -> Q GPUs: any block range of a stream decodes to the same slice of the oracle's
     reconstruction, bit for bit (ranges inside one tile, across tiles, unaligned, the tail, empty,
