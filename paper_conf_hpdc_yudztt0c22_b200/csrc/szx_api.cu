@@ -145,7 +145,8 @@ uint64_t cdiv(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
 // ------------------------------------------------------------ compress layout
 struct CLayout {
     uint64_t nB, nW, nTB, nTC;
-    uint64_t off_keys, off_zero, zero_bytes, off_scal, off_stats, off_nclist, off_nckeys, off_ncR, off_gbase, total;
+    uint64_t off_keys, off_zero, zero_bytes, off_scal, off_stats, off_nclist, off_nckeys, off_ncR, off_gbase,
+        off_codes, codes_bytes, total;
 };
 CLayout clayout(uint64_t n, int W, uint32_t b) {
     CLayout L{};
@@ -162,7 +163,9 @@ CLayout clayout(uint64_t n, int W, uint32_t b) {
     L.off_nckeys = al16(L.off_nclist + 4 * L.nB + 4);
     L.off_ncR = al16(L.off_nckeys + 2ull * W * L.nB + 16);
     L.off_gbase = al16(L.off_ncR + L.nB);
-    L.total = al16(L.off_gbase + 8 * (cdiv(L.nB, kWriteTile) + 2)) + 256;
+    L.off_codes = al16(L.off_gbase + 8 * (cdiv(L.nB, kWriteTile) + 2));
+    L.codes_bytes = (W == 4 && b == 128) ? 32 * L.nB : 0;  // lead codes, size pass -> write pass
+    L.total = al16(L.off_codes + L.codes_bytes) + 256;
     return L;
 }
 
@@ -186,6 +189,7 @@ Plan make_plan(const CLayout& L, uint8_t* ws, uint64_t n, szx_dtype_t dt, szx_eb
     p.ncmu = ws + L.off_nckeys;
     p.ncR = ws + L.off_ncR;
     p.gbase = reinterpret_cast<uint64_t*>(ws + L.off_gbase);
+    p.nccodes = L.codes_bytes ? ws + L.off_codes : nullptr;
     return p;
 }
 

@@ -53,6 +53,8 @@ struct Plan {
     void* ncmu;                // their mu (bits), same order
     uint8_t* ncR;              // classify: R_init | proven << 7; size pass: final R
     uint64_t* gbase;           // payload offset of each write tile (+ total)
+    uint8_t* nccodes;          // float32 b = 128: the 32 lead-code bytes of every full nonconstant
+                               // block (size pass -> write pass), in nonconstant order; else null
     double* eb_abs;            // [1]
     uint64_t* nnc;             // [1]
     uint64_t* total;           // [1] stream bytes (output of the call)
@@ -697,6 +699,28 @@ __device__ __forceinline__ void lane_pack_f32x8(const Lane8& e, int R, uint32_t 
     }
 }
 
+// Lead codes (16 bits, LSB-first) and mid-bytes of this lane's 8 values (size pass)
+__device__ __forceinline__ uint32_t lane_codes_f32x8(const float (&xv)[8], float mu, int R, uint32_t& msum) {
+    const int hl = threadIdx.x & 15;
+    const bool raw = R >= 32;
+    const uint32_t s = raw ? 0u : ((8u - ((uint32_t)R & 7u)) & 7u);
+    const uint32_t req = ((uint32_t)R + s) >> 3;
+    uint32_t u[8];
+#pragma unroll
+    for (int i = 0; i < 8; i++) u[i] = (raw ? __float_as_uint(xv[i]) : __float_as_uint(__fsub_rn(xv[i], mu))) >> s;
+    uint32_t prev = __shfl_up_sync(0xffffffffu, u[7], 1, 16);
+    prev = hl == 0 ? 0u : prev;
+    uint32_t leads = 0;
+    msum = 0;
+#pragma unroll
+    for (int i = 0; i < 8; i++) {
+        const uint32_t L = lead_bytes3(u[i] ^ prev);
+        prev = u[i];
+        leads |= L << (2 * i);
+        msum += req - umin_(L, req);
+    }
+    return leads;
+}
 // Mid-bytes of this lane's 8 values (size pass, half-warp per block)
 __device__ __forceinline__ uint32_t lane_msum_f32x8(const float (&xv)[8], float mu, int R) {
     const int hl = threadIdx.x & 15;
@@ -852,7 +876,9 @@ __global__ void __launch_bounds__(256) k_enc_size(const T* __restrict__ x, Plan 
                             if (!(rec1 & 0x80)) R1 = guard_R<float, 4>(x1, 4, mu1, R1, eb);
                             R = h ? R1 : R0;
                         }
-                        const uint32_t ms = lane_msum_f32x8(xv, mu, R);
+                        uint32_t ms;
+                        const uint32_t lc16 = lane_codes_f32x8(xv, mu, R, ms);
+                        reinterpret_cast<uint16_t*>(p.nccodes)[(g0 + l + h) * 16 + hl] = (uint16_t)lc16;
                         const uint32_t z0 = 33u + warp_sum(h ? 0u : ms);
                         const uint32_t z1 = 33u + warp_sum(h ? ms : 0u);
                         const uint32_t R0 = __shfl_sync(0xffffffffu, (uint32_t)R, 0);
@@ -946,10 +972,15 @@ __global__ void __launch_bounds__(256) k_enc_size(const T* __restrict__ x, Plan 
                     if constexpr (sizeof(T) == 4 && VPL == 4) {
                         if (!(rec0 & 0x80)) R0 = guard_R<T, VPL>(x0, VPL, mu0, R0, eb);
                         if (two && !(rec1 & 0x80)) R1 = guard_R<T, VPL>(x1, VPL, mu1, R1, eb);
-                        const uint32_t m0 = lane_msum_f32x4(x0, mu0, R0);
-                        const uint32_t m1 = lane_msum_f32x4(x1, mu1, R1);
-                        z0 = 33u + warp_sum(m0);
-                        if (two) z1 = 33u + warp_sum(m1);
+                        Lane4 e0, e1;
+                        lane_encode_f32x4(x0, mu0, R0, e0);
+                        lane_encode_f32x4(x1, mu1, R1, e1);
+                        p.nccodes[nc * 32 + lane] = (uint8_t)e0.leads;
+                        z0 = 33u + warp_sum(e0.msum);
+                        if (two) {
+                            p.nccodes[(nc + 1) * 32 + lane] = (uint8_t)e1.leads;
+                            z1 = 33u + warp_sum(e1.msum);
+                        }
                     } else {
                         z0 = size_block<T, VPL>(x0, mu0, R0, (rec0 & 0x80) != 0, eb);
                         z1 = two ? size_block<T, VPL>(x1, mu1, R1, (rec1 & 0x80) != 0, eb) : 0u;
@@ -981,6 +1012,7 @@ __global__ void __launch_bounds__(256) k_enc_size(const T* __restrict__ x, Plan 
                             reinterpret_cast<V*>(xv)[q] = lds_chunk<V>(st + (j + h) * C::BW + (lane * C::QV + q) * C::CB);
                         }
                         encode_block<T, VPL>(xv, VPL, B, mu, (int)(rec & 0x7F), (rec & 0x80) != 0, eb, uu, lc);
+                        if constexpr (sizeof(T) == 4 && VPL == 4) p.nccodes[(nc + h) * 32 + lane] = (uint8_t)lc.leads;
                     } else {
                         const int cnt = load_lane<T, VPL>(x, p.n, k, lane, xv);
                         const int len = (int)(p.n - (uint64_t)k * B);
@@ -1181,7 +1213,19 @@ __global__ void __launch_bounds__(256) k_enc_write(const T* __restrict__ x, Plan
                 reinterpret_cast<uint4*>(xv)[0] = lds_u128(sin + j * C::BW + hl * 32);
                 reinterpret_cast<uint4*>(xv)[1] = lds_u128(sin + j * C::BW + hl * 32 + 16);
                 Lane8 e;
-                lane_encode_f32x8(xv, cmu, R, e);
+                // lead codes from the size pass; only the shift is redone here
+                e.leads = reinterpret_cast<const uint16_t*>(p.nccodes)[(t * C::TB + bi) * 16 + hl];
+                {
+                    const bool raw = R >= 32;
+                    const uint32_t s = raw ? 0u : ((8u - ((uint32_t)R & 7u)) & 7u);
+                    const uint32_t req = ((uint32_t)R + s) >> 3;
+                    e.msum = 0;
+#pragma unroll
+                    for (int i = 0; i < 8; i++) {
+                        e.u[i] = (raw ? __float_as_uint(xv[i]) : __float_as_uint(__fsub_rn(xv[i], cmu))) >> s;
+                        e.msum += req - umin_((e.leads >> (2 * i)) & 3u, req);
+                    }
+                }
                 const uint32_t incl = half_incl_scan(e.msum);
                 lane_pack_f32x8(e, R, incl - e.msum, smem_u32(stg) + sb + zo);
             }
