@@ -473,11 +473,7 @@ __device__ inline uint32_t size_block(const T (&xv)[VPL], T mu, int& R, bool pro
 // without byte stores or run assembly.  dst is the shared-memory address of
 // the block payload; values [0, cnt) of the lane are valid, len in the block.
 __device__ inline void red_or_s(uint32_t a, uint32_t v) {
-#ifdef SZX_EXP_STS
-    asm volatile("st.shared.b32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
-#else
     asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
-#endif
 }
 __device__ inline void red_or_byte(uint32_t a, uint32_t v) { red_or_s(a & ~3u, (v & 0xFFu) << (8 * (a & 3u))); }
 
@@ -613,13 +609,8 @@ __device__ __forceinline__ uint32_t lane_msum_f32x4(const float (&xv)[4], float 
 
 // OR v into shared word a unless v == 0 (predicated, no branch)
 __device__ __forceinline__ void red_or_nz(uint32_t a, uint32_t v) {
-#ifdef SZX_EXP_STS
-    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %1, 0;\n\t@q st.shared.b32 [%0], %1;\n\t}"
-                 ::"r"(a), "r"(v) : "memory");
-#else
     asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %1, 0;\n\t@q red.shared.or.b32 [%0], %1;\n\t}"
                  ::"r"(a), "r"(v) : "memory");
-#endif
 }
 
 // ---- half-warp variants (8 values per lane, a block per 16 lanes): the

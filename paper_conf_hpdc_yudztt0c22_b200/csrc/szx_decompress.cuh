@@ -165,14 +165,8 @@ __device__ inline uint64_t cta_scan256(uint64_t v, uint64_t* agg, uint64_t* s_w 
 #ifndef SZX_DMINB
 #define SZX_DMINB 3
 #endif
-#ifndef SZX_EXP
-#define SZX_EXP 0
-#endif
 #ifndef SZX_STCS
 #define SZX_STCS 1
-#endif
-#ifndef SZX_ROT
-#define SZX_ROT 0
 #endif
 #ifndef SZX_PAIR
 #define SZX_PAIR 1   // float32 b = 128: two blocks per warp, a half-warp each
@@ -684,9 +678,6 @@ struct DecWCfg {
 #ifndef SZX_FILLW
 #define SZX_FILLW 2
 #endif
-#ifndef SZX_FSTATIC
-#define SZX_FSTATIC 0
-#endif
 #ifndef SZX_SWITCH
 #define SZX_SWITCH 2
 #endif
@@ -732,9 +723,7 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
     // index phase (the shared staging slots double as its scratch), then a
     // grid barrier: tiles are decoded by whichever warp grabs them
     index_phase<W>(p, in, hd, reinterpret_cast<uint16_t*>(dsm), s_w);
-    if (SZX_EXP & 32) return;
     grid_barrier(&p.ctr[2]);
-    if (SZX_EXP & 16) return;
     const int lane = threadIdx.x & 31;
     const uint32_t* bm = reinterpret_cast<const uint32_t*>(in + kHeaderBytes);
     const uint16_t* zs = reinterpret_cast<const uint16_t*>(in + hd.off_zs);
@@ -757,20 +746,11 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
     // retrieve with mu).  They need only the bitmap word and the tile's mu
     // values, prefetched one tile ahead, so they stream stores.
     auto fill_loop = [&]() {
-#if SZX_FSTATIC
-        uint64_t fnext = p.t_lo + ((uint64_t)blockIdx.x * C::FILLW + (threadIdx.x >> 5));
-        auto grab_f = [&]() -> uint64_t {
-            const uint64_t v = fnext;
-            fnext += (uint64_t)gridDim.x * C::FILLW;
-            return v;
-        };
-#else
         auto grab_f = [&]() -> uint64_t {
             uint32_t v = 0;
             if (lane == 0) v = atomicAdd(&p.ctr[1], 1u);
             return p.t_lo + __shfl_sync(0xffffffffu, v, 0);
         };
-#endif
         uint64_t t = grab_f();
         uint32_t word = 0;
         U mul = 0;
@@ -851,7 +831,7 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
     };
     // cp.async the segment's bytes into slot `sl`
     auto stage_seg = [&](const TileMeta<U>& m, const TileZ& z, const SegT& sg, int sl) {
-        if (!z.ok || (SZX_EXP & 8)) return;
+        if (!z.ok) return;
         const uint32_t off1 = __shfl_sync(0xffffffffu, z.zincl, sg.r1 - 1);
         const uintptr_t g0 = reinterpret_cast<uintptr_t>(pl + m.base + sg.off0);
         const uintptr_t gA = g0 & ~uintptr_t(15);
@@ -924,7 +904,7 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
         }
 #endif
 #pragma unroll 1
-        for (uint32_t bits = (SZX_EXP & 2) ? 0u : sel; bits; bits &= bits - 1) {
+        for (uint32_t bits = sel; bits; bits &= bits - 1) {
             const int j = __ffs(bits) - 1;
             const uint32_t off = __shfl_sync(0xffffffffu, offl, j);
             const uint32_t zz = __shfl_sync(0xffffffffu, zzl, j);
@@ -1029,12 +1009,10 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
         }
         cp_async_wait<0>();
     };
-    // Each warp drains its own queue first, then helps with the other one, so
-    // the split adapts to the field's fraction of nonconstant blocks.
-    if (SZX_EXP & 256) {
-        if ((int)(threadIdx.x >> 5) < C::FILLW) fill_loop();
-        return;
-    }
+    // The fill warps join the nonconstant tiles once their queue is empty, so
+    // the split adapts to the field's fraction of nonconstant blocks.  (Decode
+    // warps joining the fill as well, SZX_SWITCH = 3, measured slower: more
+    // concurrent fill streams cut the write rate -- NYX density 107 -> 149 us.)
     if ((int)(threadIdx.x >> 5) < C::FILLW) {
         fill_loop();
         if (SZX_SWITCH & 2) nc_loop();
