@@ -284,13 +284,23 @@ __global__ void __launch_bounds__(256) k_classify(Plan p, uint8_t* __restrict__ 
     uint32_t ncmask = 0;
     U rmu[8];
     uint32_t rrec[2] = {0u, 0u};  // per j: R_init | guard_proven << 7 (one byte each)
+    // all eight blocks' keys first: the stores below (mu, bitmap) could alias the
+    // stats for the compiler, which would otherwise serialise one load round trip
+    // per block
+    U kmn[8], kmx[8];
+#pragma unroll
+    for (int j = 0; j < 8; j++) {
+        const uint64_t k = base + j * 256 + threadIdx.x;
+        kmn[j] = k < p.nB ? stats[2 * k] : U(0);
+        kmx[j] = k < p.nB ? stats[2 * k + 1] : U(0);
+    }
 #pragma unroll
     for (int j = 0; j < 8; j++) {
         const uint64_t k = base + j * 256 + threadIdx.x;
         bool nc = false;
         rmu[j] = 0;
         if (k < p.nB) {
-            BlockClass<T> c = classify<T>(stats[2 * k], stats[2 * k + 1], eb);
+            BlockClass<T> c = classify<T>(kmn[j], kmx[j], eb);
             T mu = c.mu;
             if (!c.constant) {
                 nc = true;

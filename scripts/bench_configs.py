@@ -124,12 +124,29 @@ def run_case(x: torch.Tensor, eb: float, iters: int, flush: torch.Tensor | None,
             "block": b, "kernels_ms": kt, "l2_flush": flush is not None}
 
 
+def oracle_gbs(x: torch.Tensor, eb: float, b: int, reps: int = 3):
+    """Serial C oracle (1 host thread), best of `reps` compress+decompress (SURVEY 8(d) oracle
+    timing (i)); baseline only, never a code path of the product."""
+    import time
+
+    import oracle
+    arr = x.reshape(-1).cpu().numpy()
+    best = float("inf")
+    for _ in range(reps):
+        t0 = time.perf_counter()
+        s = oracle.compress(arr, eb, oracle.REL, b)
+        oracle.decompress(s)
+        best = min(best, time.perf_counter() - t0)
+    return arr.nbytes / best / 1e9
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--iters", type=int, default=20)
     ap.add_argument("--only", default="")
     ap.add_argument("--box-full", action="store_true")
     ap.add_argument("--blocks", default="128", help="block sizes to sweep, e.g. 128,256 (SURVEY 8(f) row 2)")
+    ap.add_argument("--oracle", action="store_true", help="also time the serial C oracle (configs 1-4)")
     a = ap.parse_args()
     only = set(a.only.split(",")) if a.only else None
     l2 = torch.cuda.get_device_properties(0).L2_cache_size
@@ -144,6 +161,11 @@ def main():
             for b in (int(v) for v in a.blocks.split(",")):
                 r = run_case(x, eb, a.iters, flush_buf if small else None, b)
                 r.update({"config": key, "workload": name, "eb_rel": eb, "peak_gbs": peak()})
+                if a.oracle and key != "box":
+                    g = oracle_gbs(x, eb, b)
+                    r.update({"oracle_1thread_gbs": g,
+                              "gpu_vs_oracle": (r["n"] * (4 if r["dtype"] == "f32" else 8)) /
+                              ((r["compress_ms"] + r["decompress_ms"]) * 1e6) / g})
                 print(json.dumps(r), flush=True)
         del x
         torch.cuda.empty_cache()
