@@ -21,10 +21,10 @@ if not torch.cuda.is_available():  # pragma: no cover
 import paper_conf_hpdc_yudztt0c22_b200 as szx  # noqa: E402
 
 
-def _full_parity(xd: torch.Tensor, eb: float, tag: str):
-    s = szx.compress(xd, eb, "rel", 128)
+def _full_parity(xd: torch.Tensor, eb: float, tag: str, b: int = 128):
+    s = szx.compress(xd, eb, "rel", b)
     x = xd.cpu().numpy().reshape(-1)
-    ref = oracle.compress(x, eb, oracle.REL, 128)
+    ref = oracle.compress(x, eb, oracle.REL, b)
     got = s.cpu().numpy()
     assert got.size == ref.size and got.tobytes() == ref.tobytes(), tag
     y = szx.decompress(s)
@@ -52,6 +52,13 @@ def test_config2_hurricane():
 def test_config3_nyx():
     for f in (0, 1, 2):
         _full_parity(synth.nyx_like(f, n=512, device="cuda"), 1e-3, f"nyx{f}")
+
+
+@pytest.mark.parametrize("b", [32, 64, 256])
+def test_config3_nyx_other_block_sizes(b):
+    # the block-size study at full size: dense velocity, sparse density
+    for f in (0, 1):
+        _full_parity(synth.nyx_like(f, n=512, device="cuda"), 1e-3, f"nyx{f}/b{b}", b)
 
 
 def test_config4_hacc():
