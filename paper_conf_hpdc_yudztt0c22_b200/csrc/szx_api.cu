@@ -281,8 +281,18 @@ void enqueue_encode(const void* d_in, const Plan& p, const CLayout& L, uint8_t* 
     });
     launch("k_zscan", s, [&] { launch_pdl(k_zscan<Traits<T>::W>, dim3((unsigned)L.nTC), dim3(256), 0, s, p, out); });
     using C = WriteCfg<T, VPL>;
+#ifndef SZX_WGRIDK
+#define SZX_WGRIDK 8
+#endif
+    static int occ_w = 0;
+    if (!occ_w) {
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_w, k_enc_write<T, VPL>, 256, C::SMEM);
+        if (occ_w <= 0) occ_w = 1;
+    }
+    const uint64_t wgrid = std::max<uint64_t>(1, std::min<uint64_t>(cdiv(L.nB, kWriteTile),
+                                                                    (uint64_t)SZX_WGRIDK * sm_count() * occ_w));
     launch("k_enc_write", s, [&] {
-        launch_pdl(k_enc_write<T, VPL>, dim3((unsigned)cdiv(L.nB, kWriteTile)), dim3(256), C::SMEM, s,
+        launch_pdl(k_enc_write<T, VPL>, dim3((unsigned)wgrid), dim3(256), C::SMEM, s,
                    static_cast<const T*>(d_in), p, out);
     });
 }

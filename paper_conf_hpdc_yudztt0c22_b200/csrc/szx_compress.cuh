@@ -1159,9 +1159,10 @@ __global__ void __launch_bounds__(256) k_enc_write(const T* __restrict__ x, Plan
     pdl_wait();
     pdl_trigger();
     const uint64_t nnc = *p.nnc;
-    const uint64_t t = blockIdx.x;
-    if (t * C::TB >= nnc) return;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    // tiles c, c + G, ...: the grid is capped on the host (a few CTAs per resident
+    // slot), so a sparse field does not pay for a wave of CTAs with no tile
+    for (uint64_t t = blockIdx.x; t * C::TB < nnc; t += gridDim.x) {
     const uint64_t off_zs = p.off_mu + al16((uint64_t)W * p.nB);
     const uint64_t off_pl = off_zs + al16(2 * nnc);
     const uint16_t* zsize = reinterpret_cast<const uint16_t*>(out + off_zs);
@@ -1306,6 +1307,8 @@ copy_out:
                 }
             }
         }
+    }
+    __syncthreads();  // the staging area and input buffer are reused by the next tile
     }
 }
 
