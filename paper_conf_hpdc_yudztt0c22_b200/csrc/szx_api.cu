@@ -281,6 +281,9 @@ void enqueue_encode(const void* d_in, const Plan& p, const CLayout& L, uint8_t* 
     });
     launch("k_zscan", s, [&] { launch_pdl(k_zscan<Traits<T>::W>, dim3((unsigned)L.nTC), dim3(256), 0, s, p, out); });
     using C = WriteCfg<T, VPL>;
+#ifndef SZX_ICTA_PER_SM
+#define SZX_ICTA_PER_SM 1   // decoder CTAs per SM that run the index phase
+#endif
 #ifndef SZX_WGRIDK
 #define SZX_WGRIDK 8
 #endif
@@ -472,6 +475,7 @@ int enqueue_decompress(const void* d_in, uint64_t in_bytes, const szx_header_t* 
             const uint64_t gcap = (uint64_t)sm_count() * occ;
             if (grid > gcap) grid = gcap;
             if (grid > kMaxDecodeGrid) grid = kMaxDecodeGrid;
+        p.n_icta = (uint32_t)std::min<uint64_t>(grid, (uint64_t)SZX_ICTA_PER_SM * sm_count());
             launch(name, s, [&] {
                 launch_pdl(kern, dim3((unsigned)grid), dim3(256), DecWCfg<T, V>::SMEM, s, p, in,
                            reinterpret_cast<T*>(ybase));

@@ -45,6 +45,7 @@ struct DPlan {
     uint32_t* ncpre;           // [nW]      nonconstant index of each tile's first block
     uint64_t* tbase;           // [nW + 1]  payload offset of each tile (tbase[nW] = total)
     int32_t* err;              // 0 ok, else SZX_ECORRUPT
+    uint32_t n_icta;           // CTAs that run the index phase (<= gridDim.x)
     // quality variant only: the original values, indexed
     // like y, and the accumulators {max |x-x'| (double bits), sum (x-x')^2
     // (double), dkey(min finite x), ~dkey(max finite x)}, initialised by the host
@@ -194,7 +195,7 @@ __device__ inline void stage_u16(uint16_t* s_dst, const uint16_t* __restrict__ z
 template <int W>
 __device__ inline void index_phase(const DPlan& p, const uint8_t* __restrict__ in, const DHdr& hd,
                                    uint16_t* s_zs, uint64_t* s_w) {
-    const uint64_t G = gridDim.x, c = blockIdx.x;
+    const uint64_t G = p.n_icta, c = blockIdx.x;  // the first n_icta CTAs share the index work
     const uint64_t w0 = p.nWi * c / G, w1 = p.nWi * (c + 1) / G;
     const uint32_t* bm = reinterpret_cast<const uint32_t*>(in + kHeaderBytes);
     const uint16_t* zs = reinterpret_cast<const uint16_t*>(in + hd.off_zs);
@@ -217,7 +218,7 @@ __device__ inline void index_phase(const DPlan& p, const uint8_t* __restrict__ i
         cnt += __popc(x) | (nc_tile(w, x) << 32);
     }
     const uint64_t aggP = cta_sum64(cnt, s_w);
-    const uint64_t exP = grid_excl_prefix(p.slot_a, p.res_a, &p.ctr[0], aggP, s_w);
+    const uint64_t exP = grid_excl_prefix(p.slot_a, p.res_a, &p.ctr[0], aggP, s_w, (uint32_t)G);
     const uint64_t aggA = aggP & 0xFFFFFFFFu, exA = exP & 0xFFFFFFFFu;
     uint64_t runT = exP >> 32;
     const bool ok = exA + aggA <= hd.nnc;
@@ -235,7 +236,7 @@ __device__ inline void index_phase(const DPlan& p, const uint8_t* __restrict__ i
         }
     }
     const uint64_t aggZ = cta_sum64(zsum, s_w);
-    const uint64_t exZ = grid_excl_prefix(p.slot_z, p.res_z, &p.ctr[3], aggZ, s_w);
+    const uint64_t exZ = grid_excl_prefix(p.slot_z, p.res_z, &p.ctr[3], aggZ, s_w, (uint32_t)G);
     // (3) per tile: ncpre and tbase
     uint64_t runA = exA, runZ = exZ;
     for (uint64_t wc = w0; wc < w1; wc += kIndexChunk) {
@@ -722,7 +723,8 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
     }
     // index phase (the shared staging slots double as its scratch), then a
     // grid barrier: tiles are decoded by whichever warp grabs them
-    index_phase<W>(p, in, hd, reinterpret_cast<uint16_t*>(dsm), s_w);
+    // (one CTA per SM at most: fewer arrivals at the two grid-wide prefixes)
+    if (blockIdx.x < p.n_icta) index_phase<W>(p, in, hd, reinterpret_cast<uint16_t*>(dsm), s_w);
     grid_barrier(&p.ctr[2]);
     const int lane = threadIdx.x & 31;
     const uint32_t* bm = reinterpret_cast<const uint32_t*>(in + kHeaderBytes);

@@ -379,11 +379,11 @@ __device__ inline uint64_t cta_sum64(uint64_t v, uint64_t* s_w) {
 // about three round trips, with no chained look-back and no all-to-all
 // polling.  `res` [gridDim.x] and `*arrive` must be zero.
 constexpr uint64_t kSlotFlag = 1ull << 63;
+// (over the first G CTAs of the grid; all of them must call it)
 __device__ inline uint64_t grid_excl_prefix(uint64_t* slots, uint64_t* res, uint32_t* arrive, uint64_t agg,
-                                            uint64_t* s_w /*[32]*/) {
+                                            uint64_t* s_w /*[32]*/, uint32_t G) {
     __shared__ uint32_t s_last;
     __shared__ uint64_t s_val;
-    const uint32_t G = gridDim.x;
     if (threadIdx.x == 0) {
         st_relaxed(&slots[blockIdx.x], agg);
         __threadfence();
