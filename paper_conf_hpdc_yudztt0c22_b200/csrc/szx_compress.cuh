@@ -31,9 +31,6 @@
 
 #include "szx_device.cuh"
 
-#ifndef SZX_WPAIR
-#define SZX_WPAIR 1   // size and write passes: two float32 blocks per warp, a half-warp each
-#endif
 
 namespace szx {
 
@@ -851,7 +848,6 @@ __global__ void __launch_bounds__(256) k_enc_size(const T* __restrict__ x, Plan 
                     }
                     __syncwarp();
                     const uint32_t st = sbuf + (b & 1) * C::NB * C::BW;
-#if SZX_WPAIR
                     // two blocks at once, a half-warp each (8 values per lane)
 #pragma unroll
                     for (int j = 0; j < C::NB; j += 2) {
@@ -889,30 +885,6 @@ __global__ void __launch_bounds__(256) k_enc_size(const T* __restrict__ x, Plan 
                         zr = lane == l + 1 ? z1 : zr;
                         rr = lane == l + 1 ? R1 : rr;
                     }
-#else
-#pragma unroll
-                    for (int j = 0; j < C::NB; j += 2) {
-                        const int l = b * C::NB + j;
-                        float x0[4], x1[4];
-                        reinterpret_cast<uint4*>(x0)[0] = lds_u128(st + j * C::BW + lane * 16);
-                        reinterpret_cast<uint4*>(x1)[0] = lds_u128(st + (j + 1) * C::BW + lane * 16);
-                        const float mu0 = __uint_as_float(__shfl_sync(0xffffffffu, (uint32_t)mmu, l));
-                        const float mu1 = __uint_as_float(__shfl_sync(0xffffffffu, (uint32_t)mmu, l + 1));
-                        const uint32_t rec0 = __shfl_sync(0xffffffffu, mrec, l);
-                        const uint32_t rec1 = __shfl_sync(0xffffffffu, mrec, l + 1);
-                        int R0 = (int)(rec0 & 0x7F), R1 = (int)(rec1 & 0x7F);
-                        if (!(rec0 & rec1 & 0x80)) {  // a block whose R2 check was not proven away
-                            if (!(rec0 & 0x80)) R0 = guard_R<float, 4>(x0, 4, mu0, R0, eb);
-                            if (!(rec1 & 0x80)) R1 = guard_R<float, 4>(x1, 4, mu1, R1, eb);
-                        }
-                        const uint32_t z0 = 33u + warp_sum(lane_msum_f32x4(x0, mu0, R0));
-                        const uint32_t z1 = 33u + warp_sum(lane_msum_f32x4(x1, mu1, R1));
-                        zr = lane == l ? z0 : zr;
-                        rr = lane == l ? (uint32_t)R0 : rr;
-                        zr = lane == l + 1 ? z1 : zr;
-                        rr = lane == l + 1 ? (uint32_t)R1 : rr;
-                    }
-#endif
                     __syncwarp();
                 }
                 zsize[gi] = (uint16_t)zr;
@@ -1199,9 +1171,9 @@ __global__ void __launch_bounds__(256) k_enc_write(const T* __restrict__ x, Plan
     }
     cp_async_wait<0>();
     __syncthreads();
+    bool packed = false;
     if constexpr (sizeof(T) == 4 && VPL == 4) {
         if (tfull) {  // branch-free body: every block of the tile is a full float32 block
-#if SZX_WPAIR
             // two blocks per step, a half-warp each (8 values per lane)
             const int h = lane >> 4, hl = lane & 15;
 #pragma unroll
@@ -1231,24 +1203,10 @@ __global__ void __launch_bounds__(256) k_enc_write(const T* __restrict__ x, Plan
                 const uint32_t incl = half_incl_scan(e.msum);
                 lane_pack_f32x8(e, R, incl - e.msum, smem_u32(stg) + sb + zo);
             }
-            goto copy_out;
-#endif
-#pragma unroll
-            for (int j = 0; j < C::BPW; j++) {
-                const int bi = warp * C::BPW + j;
-                const uint32_t zo = __shfl_sync(0xffffffffu, zincl - zl, bi);
-                const float cmu = __uint_as_float(__shfl_sync(0xffffffffu, (uint32_t)mmu, j));
-                const int R = (int)__shfl_sync(0xffffffffu, mR, j);
-                float xv[4];
-                reinterpret_cast<uint4*>(xv)[0] = lds_u128(sin + j * C::BW + lane * 16);
-                Lane4 e;
-                lane_encode_f32x4(xv, cmu, R, e);
-                const uint32_t incl = warp_incl_scan(e.msum);
-                lane_pack_f32x4(e, R, incl - e.msum, smem_u32(stg) + sb + zo);
-            }
-            goto copy_out;
+            packed = true;
         }
     }
+    if (!packed) {
 #pragma unroll 1
     for (int j = 0; j < C::BPW; j++) {
         const int bi = warp * C::BPW + j;
@@ -1283,7 +1241,7 @@ __global__ void __launch_bounds__(256) k_enc_write(const T* __restrict__ x, Plan
             pack_red<T, VPL>(u, lc, cnt, len, smem_u32(stg) + sb + zo);
         }
     }
-copy_out:
+    }
     __syncthreads();
     // copy the staged tile payload to global memory with 16-byte stores
     uint8_t* g0 = out + off_pl + base;

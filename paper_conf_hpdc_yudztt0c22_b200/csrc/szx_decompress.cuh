@@ -169,9 +169,6 @@ __device__ inline uint64_t cta_scan256(uint64_t v, uint64_t* agg, uint64_t* s_w 
 #ifndef SZX_STCS
 #define SZX_STCS 1
 #endif
-#ifndef SZX_PAIR
-#define SZX_PAIR 1   // float32 b = 128: two blocks per warp, a half-warp each
-#endif
 constexpr int kIndexChunk = 256;
 
 // Copy zs[i0, i0 + cnt) (cnt <= 32 * kIndexChunk) into shared memory with
@@ -869,7 +866,6 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
         const uint32_t sel = __ballot_sync(0xffffffffu, insg) & rm;
         const uint32_t offl = __shfl_sync(0xffffffffu, z.zincl - z.zl, rank);
         const uint32_t zzl = __shfl_sync(0xffffffffu, z.zl, rank);
-#if SZX_PAIR
         if constexpr (sizeof(T) == 4 && VPL == 4) {
             // two blocks per iteration, a half-warp each (the second half idles
             // on the last block of an odd count)
@@ -902,25 +898,24 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
                     }
                 }
             }
-            return;
-        }
-#endif
+        } else {
 #pragma unroll 1
-        for (uint32_t bits = sel; bits; bits &= bits - 1) {
-            const int j = __ffs(bits) - 1;
-            const uint32_t off = __shfl_sync(0xffffffffu, offl, j);
-            const uint32_t zz = __shfl_sync(0xffffffffu, zzl, j);
-            const T mu = TR::from(__shfl_sync(0xffffffffu, m.mul, j));
-            T v[VPL];
-            if (!decode_full_g<T, VPL>(SrcS{sbase + off}, zz, mu, v)) {
-                if (lane == 0) set_corrupt(p.err);
-                continue;
-            }
+            for (uint32_t bits = sel; bits; bits &= bits - 1) {
+                const int j = __ffs(bits) - 1;
+                const uint32_t off = __shfl_sync(0xffffffffu, offl, j);
+                const uint32_t zz = __shfl_sync(0xffffffffu, zzl, j);
+                const T mu = TR::from(__shfl_sync(0xffffffffu, m.mul, j));
+                T v[VPL];
+                if (!decode_full_g<T, VPL>(SrcS{sbase + off}, zz, mu, v)) {
+                    if (lane == 0) set_corrupt(p.err);
+                    continue;
+                }
 #pragma unroll
-            for (int q = 0; q < NV; q++) st_out(yq + j * QB + q, reinterpret_cast<const V*>(v)[q]);
-            if constexpr (QUAL)
-                qa.add16<T, NV, V>(reinterpret_cast<const V*>(ref + t * TB * B + lane * VPL) + j * QB,
-                                   reinterpret_cast<const V(&)[NV]>(v));
+                for (int q = 0; q < NV; q++) st_out(yq + j * QB + q, reinterpret_cast<const V*>(v)[q]);
+                if constexpr (QUAL)
+                    qa.add16<T, NV, V>(reinterpret_cast<const V*>(ref + t * TB * B + lane * VPL) + j * QB,
+                                       reinterpret_cast<const V(&)[NV]>(v));
+            }
         }
     };
     // the partial last tile: generic decoder, straight from global memory
