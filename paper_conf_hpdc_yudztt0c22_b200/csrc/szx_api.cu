@@ -1152,4 +1152,11 @@ const char* szx_strerror(int code) {
     }
 }
 
+#if SZX_TIMELINE
+// diagnostic timing builds only: copy the decoder's per-warp timeline to host
+int szx_debug_timeline(uint64_t* h_dst, uint64_t n) {
+    const uint64_t cap = sizeof(szx::g_tl) / sizeof(uint64_t);
+    return cudaMemcpyFromSymbol(h_dst, szx::g_tl, 8 * (n < cap ? n : cap)) == cudaSuccess ? SZX_OK : SZX_ECUDA;
+}
+#endif
 }  // extern "C"

@@ -684,6 +684,29 @@ struct DecWCfg {
     static_assert(SMEM >= kIndexChunk * 32 * 2, "index-phase scratch aliases the slots");
 };
 
+// Diagnostic timing builds only (-DSZX_TIMELINE=1, scripts/timeline.py): per
+// warp of k_decode_w, %globaltimer at kernel entry, index ready, fill done,
+// nonconstant tiles done.
+#ifndef SZX_TIMELINE
+#define SZX_TIMELINE 0
+#endif
+#if SZX_TIMELINE
+constexpr int kTlCtas = 2048;
+__device__ uint64_t g_tl[kTlCtas * 8 * 4];
+#define SZX_TL(k)                                                                                 \
+    do {                                                                                          \
+        if ((threadIdx.x & 31) == 0 && blockIdx.x < kTlCtas) {                                    \
+            uint64_t t_;                                                                          \
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_) : : "memory");                   \
+            g_tl[((uint64_t)blockIdx.x * 8 + (threadIdx.x >> 5)) * 4 + (k)] = t_;                 \
+        }                                                                                         \
+    } while (0)
+#else
+#define SZX_TL(k) \
+    do {          \
+    } while (0)
+#endif
+
 // Per-tile metadata a warp needs before it can store anything.
 template <typename U>
 struct TileMeta {
@@ -713,6 +736,7 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
     const T* __restrict__ ref = static_cast<const T*>(p.ref);
     pdl_wait();
     pdl_trigger();
+    SZX_TL(0);
     const DHdr hd = read_dheader<W>(in, p);
     if (!hd.ok) {  // every CTA sees the same header: all leave
         if (blockIdx.x == 0 && threadIdx.x == 0) set_corrupt(p.err);
@@ -723,6 +747,7 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
     // (one CTA per SM at most: fewer arrivals at the two grid-wide prefixes)
     if (blockIdx.x < p.n_icta) index_phase<W>(p, in, hd, reinterpret_cast<uint16_t*>(dsm), s_w);
     grid_barrier(&p.ctr[2]);
+    SZX_TL(1);
     const int lane = threadIdx.x & 31;
     const uint32_t* bm = reinterpret_cast<const uint32_t*>(in + kHeaderBytes);
     const uint16_t* zs = reinterpret_cast<const uint16_t*>(in + hd.off_zs);
@@ -1012,11 +1037,13 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
     // concurrent fill streams cut the write rate -- NYX density 107 -> 149 us.)
     if ((int)(threadIdx.x >> 5) < C::FILLW) {
         fill_loop();
+        SZX_TL(2);
         if (SZX_SWITCH & 2) nc_loop();
     } else {
         nc_loop();
         if (SZX_SWITCH & 1) fill_loop();
     }
+    SZX_TL(3);
     if constexpr (QUAL) qa.flush(p.qual);
 }
 
