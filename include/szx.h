@@ -252,6 +252,28 @@ int szx_compress_shard_async(const void* d_in, szx_dtype_t dt, uint64_t n, szx_e
                              void* d_out, uint64_t out_capacity, void* d_ws, uint64_t ws_bytes,
                              uint64_t* d_total_bytes, void* stream);
 
+/* SURVEY 8(b)'s double-valued forms of the two sharded passes (thin wrappers
+ * over the key-based calls above).
+ *
+ * szx_local_minmax: the finite-value range of the shard, d_minmax2[0] = min,
+ * d_minmax2[1] = max as doubles (exact widening of the data type; -0 and +0
+ * compare as -0 < +0, reading R13); no finite value -> (+Inf, -Inf).  Combine
+ * shards with an all-reduce MIN of [0] and MAX of [1]; then
+ * eb_abs = REL x (max - min) in double (footnote 1).  Non-blocking
+ * (stream-ordered scratch).  Returns SZX_OK / SZX_EINVAL / SZX_ECUDA /
+ * SZX_ENOMEM. */
+int szx_local_minmax(const void* d_in, szx_dtype_t dt, uint64_t n, double* d_minmax2, void* stream);
+
+/* szx_compress_shard: compress the shard as a standalone SZX1 stream whose
+ * absolute bound is *d_eb_abs (device double, e.g. computed from the
+ * all-reduced szx_local_minmax); the header records mode and eb_user as given
+ * and eb_abs.  Byte-identical to the oracle's orc_compress_shard with the same
+ * eb_abs.  Blocking: returns the stream bytes, or SZX_EINVAL / SZX_ENOSPC
+ * (out_capacity < szx_compress_bound) / SZX_ECUDA / SZX_ENOMEM. */
+int64_t szx_compress_shard(const void* d_in, szx_dtype_t dt, uint64_t n, szx_ebmode_t mode, double eb_user,
+                           const double* d_eb_abs, uint32_t block_size, void* d_out, uint64_t out_capacity,
+                           void* stream);
+
 /* ------------------------------------------------------------ diagnostics */
 
 /* Per-kernel device timing with CUDA events recorded on the launch stream

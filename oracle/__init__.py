@@ -36,7 +36,60 @@ def build(force: bool = False) -> str:
     return _LIB
 
 
+_OMP_SRC = os.path.join(_HERE, "szx_omp.c")
+_OMP_LIB = os.path.join(_HERE, "libszx_omp.so")
+
+
+def build_omp(force: bool = False) -> str:
+    """Compile the OpenMP-design host baseline (szx_omp.c includes szx_oracle.c; same FP flags)."""
+    if (force or not os.path.exists(_OMP_LIB)
+            or os.path.getmtime(_OMP_LIB) < max(os.path.getmtime(_OMP_SRC), os.path.getmtime(_SRC))):
+        tmp = _OMP_LIB + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", *CFLAGS, "-fopenmp", "-o", tmp, _OMP_SRC, "-lm"], cwd=_HERE)
+        os.replace(tmp, _OMP_LIB)
+    return _OMP_LIB
+
+
 _lib = None
+_omp = None
+
+
+def omp_lib():
+    global _omp
+    if _omp is None:
+        build_omp()
+        L = ctypes.CDLL(_OMP_LIB)
+        L.omp_compress.restype = ctypes.c_int64
+        L.omp_compress.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.c_uint64, ctypes.c_int, ctypes.c_double,
+                                   ctypes.c_uint32, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int]
+        L.omp_decompress.restype = ctypes.c_int64
+        L.omp_decompress.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_uint64,
+                                     ctypes.c_int]
+        _omp = L
+    return _omp
+
+
+def omp_compress(x: np.ndarray, eb: float, mode: int = REL, b: int = 128, threads: int = 0) -> np.ndarray:
+    """The paper's OpenMP design (Sec. 6.1): one stream, byte-identical to compress()."""
+    x = np.ascontiguousarray(x).reshape(-1)
+    dt = _dtype_code(x)
+    out = np.empty(max(compress_bound(x.size, dt, b), 64), dtype=np.uint8)
+    r = omp_lib().omp_compress(x.ctypes.data if x.size else None, dt, x.size, mode, float(eb), b,
+                               out.ctypes.data, out.size, int(threads))
+    if r < 0:
+        raise ValueError(f"omp_compress failed: {r}")
+    return out[:r].copy()
+
+
+def omp_decompress(stream: np.ndarray, threads: int = 0) -> np.ndarray:
+    stream = np.ascontiguousarray(stream, dtype=np.uint8)
+    h = read_header(stream)
+    out = np.empty(h["n"], dtype=np.float32 if h["dtype"] == F32 else np.float64)
+    r = omp_lib().omp_decompress(stream.ctypes.data, stream.size, out.ctypes.data if out.size else None,
+                                 out.nbytes, int(threads))
+    if r < 0:
+        raise ValueError(f"omp_decompress failed: {r}")
+    return out
 
 
 def lib():

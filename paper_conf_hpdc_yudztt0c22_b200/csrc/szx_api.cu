@@ -8,6 +8,7 @@
 #include <atomic>
 #include <cmath>
 #include <cstring>
+#include <map>
 #include <mutex>
 #include <vector>
 
@@ -20,6 +21,10 @@ using namespace szx;
 namespace {
 
 constexpr uint64_t kMaxN = 1ull << 36;
+// the decoder's index phase packs a block count and a tile count into the two
+// 32-bit halves of one u64 (szx_decompress.cuh, index_phase); the smallest
+// block size (32) bounds the block count
+static_assert(kMaxN / 32 < (1ull << 32), "block counts must fit 32 bits");
 
 std::atomic<uint64_t> g_launches{0};
 std::atomic<int> g_rbias{0};
@@ -90,6 +95,29 @@ void launch_pdl(void (*k)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStr
     at[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = at;
     cfg.numAttrs = timing_on() ? 0 : 1;
+    cudaLaunchKernelEx(&cfg, k, static_cast<KArgs>(args)...);
+}
+
+// Cooperative launch (co-residency guaranteed by the driver or the launch
+// fails) for the persistent kernels that spin on other CTAs' flags, combined
+// with PDL when the driver accepts both attributes; otherwise cooperative only.
+template <typename... KArgs, typename... Args>
+void launch_coop(void (*k)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s, Args... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute at[2];
+    at[0].id = cudaLaunchAttributeCooperative;
+    at[0].val.cooperative = 1;
+    at[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[1].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = timing_on() ? 1 : 2;
+    if (cudaLaunchKernelEx(&cfg, k, static_cast<KArgs>(args)...) == cudaSuccess) return;
+    cudaGetLastError();
+    cfg.numAttrs = 1;
     cudaLaunchKernelEx(&cfg, k, static_cast<KArgs>(args)...);
 }
 
@@ -221,35 +249,55 @@ constexpr int stats_unroll() {
     return u < 1 ? 1 : (u > 16 ? 16 : u);
 }
 
-template <typename T, int VPL>
-void set_smem_attrs() {
-    static bool done = false;
-    if (done) return;
-    constexpr int UNR = stats_unroll<T, VPL>();
-    carve(k_block_stats<T, VPL, UNR>);
-    carve(k_classify<T>);
-    carve(k_enc_size<T, VPL>);
-    carve(k_zscan<Traits<T>::W>);
-    carve(k_enc_write<T, VPL>);
-    carve(k_decode_w<T, VPL>);
-    carve(k_decode_w<T, VPL, true>);
-    cudaFuncSetAttribute(k_enc_write<T, VPL>, cudaFuncAttributeMaxDynamicSharedMemorySize, WriteCfg<T, VPL>::SMEM);
-    cudaFuncSetAttribute(k_enc_size<T, VPL>, cudaFuncAttributeMaxDynamicSharedMemorySize, SizeCfg<T, VPL>::SMEM);
+// Per-device kernel set-up.  Function attributes (dynamic shared memory limit,
+// carve-out) belong to the device context, and the occupancy that sizes the
+// persistent grids is a property of the device, so both are cached per
+// (device, kernel, dynamic smem), under a mutex (callers may be several host
+// threads, each driving its own device).
+struct KernelSetup {
+    std::mutex mu;
+    struct Key {
+        int dev;
+        const void* fn;
+        size_t smem;
+        bool operator<(const Key& o) const {
+            if (dev != o.dev) return dev < o.dev;
+            if (fn != o.fn) return fn < o.fn;
+            return smem < o.smem;
+        }
+    };
+    std::map<Key, int> occ;
+};
+KernelSetup& kernel_setup() { static KernelSetup k; return k; }
 
-    done = true;
+// Blocks of `k` per SM at 256 threads with `smem` dynamic bytes on the current
+// device (attributes set on first use per device); `dflt` if the query fails.
+template <typename K>
+int kernel_occupancy(K k, size_t smem, int dflt) {
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return dflt; }
+    KernelSetup& S = kernel_setup();
+    std::lock_guard<std::mutex> g(S.mu);
+    const KernelSetup::Key key{dev, reinterpret_cast<const void*>(k), smem};
+    auto it = S.occ.find(key);
+    if (it != S.occ.end()) return it->second;
+    carve(k);
+    if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    int occ = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, 256, smem) != cudaSuccess || occ <= 0) {
+        cudaGetLastError();
+        occ = dflt;
+    }
+    S.occ[key] = occ;
+    return occ;
 }
 
 // grid-stride streaming pass: enough CTAs to fill every SM, each warp keeping
 // UNR blocks (128 bytes per lane) of loads in flight
 template <typename T, int VPL>
 void enqueue_stats(const void* d_in, const Plan& p, int want_range, cudaStream_t s) {
-    set_smem_attrs<T, VPL>();
     constexpr int UNR = stats_unroll<T, VPL>();
-    static int occ = 0;
-    if (!occ) {
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_block_stats<T, VPL, UNR>, 256, 0);
-        if (occ <= 0) occ = 4;
-    }
+    const int occ = kernel_occupancy(k_block_stats<T, VPL, UNR>, 0, 4);
     uint64_t grid = cdiv(p.nB, 8 * UNR);
     const uint64_t cap = (uint64_t)sm_count() * occ;
     if (grid > cap) grid = cap;
@@ -264,13 +312,10 @@ void enqueue_stats(const void* d_in, const Plan& p, int want_range, cudaStream_t
 // nonconstant); CTAs beyond the device-side count exit at once.
 template <typename T, int VPL>
 void enqueue_encode(const void* d_in, const Plan& p, const CLayout& L, uint8_t* out, cudaStream_t s) {
-    set_smem_attrs<T, VPL>();
+    kernel_occupancy(k_classify<T>, 0, 1);
+    kernel_occupancy(k_zscan<Traits<T>::W>, 0, 1);
     launch("k_classify", s, [&] { launch_pdl(k_classify<T>, dim3((unsigned)L.nTB), dim3(256), 0, s, p, out); });
-    static int occ = 0;
-    if (!occ) {
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_enc_size<T, VPL>, 256, SizeCfg<T, VPL>::SMEM);
-        if (occ <= 0) occ = 2;
-    }
+    const int occ = kernel_occupancy(k_enc_size<T, VPL>, SizeCfg<T, VPL>::SMEM, 2);
     uint64_t grid = cdiv(L.nB, 8);
     const uint64_t cap = (uint64_t)sm_count() * occ;
     if (grid > cap) grid = cap;
@@ -287,11 +332,7 @@ void enqueue_encode(const void* d_in, const Plan& p, const CLayout& L, uint8_t* 
 #ifndef SZX_WGRIDK
 #define SZX_WGRIDK 8
 #endif
-    static int occ_w = 0;
-    if (!occ_w) {
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_w, k_enc_write<T, VPL>, 256, C::SMEM);
-        if (occ_w <= 0) occ_w = 1;
-    }
+    const int occ_w = kernel_occupancy(k_enc_write<T, VPL>, C::SMEM, 1);
     const uint64_t wgrid = std::max<uint64_t>(1, std::min<uint64_t>(cdiv(L.nB, kWriteTile),
                                                                     (uint64_t)SZX_WGRIDK * sm_count() * occ_w));
     launch("k_enc_write", s, [&] {
@@ -462,28 +503,25 @@ int enqueue_decompress(const void* d_in, uint64_t in_bytes, const szx_header_t* 
     dispatch((szx_dtype_t)h->dtype, h->block_size, [&](auto tag, auto vpl) {
         using T = decltype(tag);
         constexpr int V = decltype(vpl)::value;
-        set_smem_attrs<T, V>();
         // persistent, co-resident grid (index phase, grid barrier, then one
-        // warp per 32-block tile)
-        auto go = [&](auto kern, int& occ, const char* name) {
-            if (!occ) {
-                cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, DecWCfg<T, V>::SMEM);
-                cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, 256, DecWCfg<T, V>::SMEM);
-                if (occ <= 0) occ = 2;
-            }
+        // warp per 32-block tile): launched cooperatively, so the driver
+        // either makes every CTA resident at once or rejects the launch (it
+        // never hangs when fewer SMs are available, e.g. under MPS limits or
+        // beside a concurrent kernel)
+        auto go = [&](auto kern, const char* name) {
+            const int occ = kernel_occupancy(kern, DecWCfg<T, V>::SMEM, 1);
             uint64_t grid = cdiv(p.nWi, 8);
             const uint64_t gcap = (uint64_t)sm_count() * occ;
             if (grid > gcap) grid = gcap;
             if (grid > kMaxDecodeGrid) grid = kMaxDecodeGrid;
-        p.n_icta = (uint32_t)std::min<uint64_t>(grid, (uint64_t)SZX_ICTA_PER_SM * sm_count());
+            p.n_icta = (uint32_t)std::min<uint64_t>(grid, (uint64_t)SZX_ICTA_PER_SM * sm_count());
             launch(name, s, [&] {
-                launch_pdl(kern, dim3((unsigned)grid), dim3(256), DecWCfg<T, V>::SMEM, s, p, in,
-                           reinterpret_cast<T*>(ybase));
+                launch_coop(kern, dim3((unsigned)grid), dim3(256), DecWCfg<T, V>::SMEM, s, p, in,
+                            reinterpret_cast<T*>(ybase));
             });
         };
-        static int occ = 0, occ_q = 0;
-        if (d_ref) go(k_decode_w<T, V, true>, occ_q, "k_decode_q");
-        else go(k_decode_w<T, V>, occ, "k_decode");
+        if (d_ref) go(k_decode_w<T, V, true>, "k_decode_q");
+        else go(k_decode_w<T, V>, "k_decode");
     });
     return cudaGetLastError() == cudaSuccess ? SZX_OK : SZX_ECUDA;
 }
@@ -817,7 +855,7 @@ int64_t szx_decompress_host(const void* h_in, uint64_t in_bytes, void* h_out, ui
             if (in_bytes >= 32 + 32 + 64) {
                 uint64_t off;
                 memcpy(&off, hb + 32 + 16, 8);
-                if (off + 64 <= in_bytes) W = hb[off + 5] ? 8 : 4;
+                if (off <= in_bytes && in_bytes - off >= 64) W = hb[off + 5] ? 8 : 4;
             }
         } else {
             szx_header_t h;
@@ -887,6 +925,74 @@ int szx_compress_shard_async(const void* d_in, szx_dtype_t dt, uint64_t n, szx_e
     return cudaGetLastError() == cudaSuccess ? SZX_OK : SZX_ECUDA;
 }
 
+}  // extern "C"
+
+// keys [key(min), ~key(max)] -> doubles (min, max); no finite value -> (+Inf, -Inf)
+__global__ void k_keys_to_minmax(const uint64_t* keys, double* mm) {
+    const uint64_t a = keys[0], c = keys[1];
+    mm[0] = a == ~0ull ? __longlong_as_double(0x7FF0000000000000ll) : __longlong_as_double((long long)dkey_inv(a));
+    mm[1] = c == ~0ull ? __longlong_as_double((long long)0xFFF0000000000000ull)
+                       : __longlong_as_double((long long)dkey_inv(~c));
+}
+
+extern "C" {
+
+int szx_local_minmax(const void* d_in, szx_dtype_t dt, uint64_t n, double* d_minmax2, void* stream) {
+    if (dt != SZX_F32 && dt != SZX_F64) return SZX_EINVAL;
+    if (!d_minmax2 || (n && (!d_in || !aligned16(d_in))) || n > kMaxN) return SZX_EINVAL;
+    if (!have_device()) return SZX_ECUDA;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    const uint64_t wsb = std::max<uint64_t>(szx_compress_workspace_bytes(n, dt, 128), 16) + 16;
+    void* ws = nullptr;
+    keep_pool_memory();
+    if (cudaMallocAsync(&ws, wsb, s) != cudaSuccess) { cudaGetLastError(); return SZX_ENOMEM; }
+    uint64_t* keys = reinterpret_cast<uint64_t*>(static_cast<uint8_t*>(ws) + wsb - 16);
+    int rc = szx_local_range(d_in, dt, n, 128, keys, ws, wsb - 16, stream);
+    if (rc == SZX_OK) {
+        launch("k_keys_to_minmax", s, [&] { k_keys_to_minmax<<<1, 1, 0, s>>>(keys, d_minmax2); });
+        rc = cudaGetLastError() == cudaSuccess ? SZX_OK : SZX_ECUDA;
+    }
+    cudaFreeAsync(ws, s);
+    return rc;
+}
+
+int64_t szx_compress_shard(const void* d_in, szx_dtype_t dt, uint64_t n, szx_ebmode_t mode, double eb_user,
+                           const double* d_eb_abs, uint32_t b, void* d_out, uint64_t cap, void* stream) {
+    int rc = check_compress_args(d_in, dt, n, mode, eb_user, b, d_out);
+    if (rc) return rc;
+    if (!d_eb_abs) return SZX_EINVAL;
+    if (!have_device()) return SZX_ECUDA;
+    if (cap < szx_compress_bound(n, dt, b)) return SZX_ENOSPC;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    const int W = wbytes(dt);
+    CLayout L = clayout(n, W, b);
+    void* wsv = nullptr;
+    keep_pool_memory();
+    if (cudaMallocAsync(&wsv, L.total, s) != cudaSuccess) { cudaGetLastError(); return SZX_ENOMEM; }
+    uint8_t* ws = static_cast<uint8_t*>(wsv);
+    uint8_t* out = static_cast<uint8_t*>(d_out);
+    Plan p = make_plan(L, ws, n, dt, mode, eb_user, b, nullptr);
+    p.eb_in = d_eb_abs;
+    if (n == 0) {
+        launch("k_empty_header", s, [&] {
+            k_empty_header<<<1, 1, 0, s>>>(out, dt, mode, b, eb_user, nullptr, p.total, d_eb_abs);
+        });
+    } else {
+        cudaMemsetAsync(ws + L.off_keys, 0xFF, 16, s);
+        cudaMemsetAsync(ws + L.off_zero, 0, L.zero_bytes, s);
+        dispatch(dt, b, [&](auto tag, auto vpl) {
+            using T = decltype(tag);
+            constexpr int V = decltype(vpl)::value;
+            enqueue_stats<T, V>(d_in, p, 0, s);
+            enqueue_encode<T, V>(d_in, p, L, out, s);
+        });
+    }
+    int64_t r = SZX_ECUDA;
+    uint64_t total = 0;
+    if (cudaGetLastError() == cudaSuccess && finish_sync(s, p.total, &total) == SZX_OK) r = (int64_t)total;
+    cudaFreeAsync(wsv, s);
+    return r;
+}
 
 // ------------------------------------------------------------ dump / load
 // Single-box analogue of the paper's data dumping / loading experiment

@@ -42,6 +42,7 @@ struct Plan {
     double eb_user;
     // workspace
     uint64_t* range_keys;      // [2] finite range keys (min, ~max), init 0xFF..
+    const double* eb_in;       // non-null: the absolute bound, given (szx_compress_shard)
     uint32_t* ctr;             // [4] tile tickets, init 0
     uint64_t* status_b;        // classify look-back, init 0
     uint64_t* status_c;        // encode look-back, init 0
@@ -272,7 +273,7 @@ __global__ void __launch_bounds__(256) k_classify(Plan p, uint8_t* __restrict__ 
     const uint64_t tile = s_tile;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const uint64_t base = tile * kClassifyBlocks;
-    const double eb = eb_from_range(p.mode, p.eb_user, p.range_keys);
+    const double eb = eb_from_range(p.mode, p.eb_user, p.range_keys, p.eb_in);
     const int pe = expo_f64(eb);
     const U* stats = reinterpret_cast<const U*>(p.stats);
     uint32_t* bitmap = reinterpret_cast<uint32_t*>(out + kHeaderBytes);
@@ -1271,14 +1272,14 @@ __global__ void __launch_bounds__(256) k_enc_write(const T* __restrict__ x, Plan
 }
 
 __global__ void k_empty_header(uint8_t* out, uint32_t dtype, uint32_t mode, uint32_t b, double eb_user,
-                               const uint64_t* range_keys, uint64_t* total) {
+                               const uint64_t* range_keys, uint64_t* total, const double* eb_in = nullptr) {
     uint64_t* h = reinterpret_cast<uint64_t*>(out);
     h[0] = 0x31585A53ull | (1ull << 32) | ((uint64_t)dtype << 40) | ((uint64_t)mode << 48);
     h[1] = b;
     h[2] = 0;
     h[3] = (uint64_t)__double_as_longlong(eb_user);
     // REL: the (global) range of a sharded array, or no values at all -> 0
-    const double e = eb_from_range(mode, eb_user, range_keys);
+    const double e = eb_from_range(mode, eb_user, range_keys, eb_in);
     h[4] = (uint64_t)__double_as_longlong(e);
     h[5] = 0;
     h[6] = 0;

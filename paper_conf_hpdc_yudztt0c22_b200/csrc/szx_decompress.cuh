@@ -164,10 +164,13 @@ __device__ inline uint64_t cta_scan256(uint64_t v, uint64_t* agg, uint64_t* s_w 
 // starting nonconstant index and payload offset; it then scans its range in
 // chunks of 256 tiles.  Run by all 256 threads; s_zs: 256*32 u16 scratch.
 #ifndef SZX_DMINB
-#define SZX_DMINB 3
+#define SZX_DMINB (SZX_DQUARTER ? 2 : 3)  // decoder CTAs per SM (register budget of the block decoder)
 #endif
 #ifndef SZX_STCS
 #define SZX_STCS 1
+#endif
+#ifndef SZX_DQUARTER
+#define SZX_DQUARTER 0   // float32 b = 128: quarter-warp (1) or half-warp (0) block decoder
 #endif
 constexpr int kIndexChunk = 256;
 
@@ -208,7 +211,8 @@ __device__ inline void index_phase(const DPlan& p, const uint8_t* __restrict__ i
         return ((word != 0u || w >= nW_full) && w >= p.t_lo) ? 1u : 0u;
     };
     // (1) nonconstant blocks (low 32 bits) and such tiles (high 32 bits) in the
-    // range -> starting nonconstant index and list position.  nNC <= 2^29.
+    // range -> starting nonconstant index and list position.  Both fit 32 bits:
+    // nB <= kMaxN / 32 = 2^31 (static_assert beside kMaxN in szx_api.cu).
     uint64_t cnt = 0;
     for (uint64_t w = w0 + threadIdx.x; w < w1; w += kIndexChunk) {
         const uint32_t x = word_at(w);
@@ -576,6 +580,100 @@ __device__ __forceinline__ bool decode_half_f32x8(uint32_t a, uint32_t z, float 
     return ok;
 }
 
+// ---- four float32 blocks of b = 128 per warp: a quarter-warp (8 lanes) per
+// block, 16 values per lane.  Fig. 10's five steps as in
+// decode_half_f32x8; the per-lane steps (R and code parsing, the mid-byte
+// scan, the lead-byte map scan, the z check) are paid once per 16 values and
+// the scans take three shuffle steps.  Shifts by the block constants drop and
+// s are multiplications by powers of two (FMA pipe), so the integer ALU only
+// sees the per-value extract / mask / select work.  Non-raw blocks only
+// (9 <= R < 32): the caller routes raw or malformed blocks to the generic path.
+template <int O>
+__device__ __forceinline__ uint32_t shfl_up_add8(uint32_t v) {
+    asm volatile(
+        "{\n\t.reg .u32 t;\n\t.reg .pred p;\n\t"
+        "shfl.sync.up.b32 t|p, %0, %1, 0x1800, -1;\n\t"
+        "@p add.u32 %0, %0, t;\n\t}"
+        : "+r"(v)
+        : "n"(O));
+    return v;
+}
+// quarter q decodes the block whose payload starts at shared address a (z
+// bytes, R read by the caller); returns false (whole quarter) on a malformed block
+__device__ __forceinline__ bool decode_quarter_f32x16(uint32_t a, uint32_t R, uint32_t z, float mu,
+                                                      float (&out)[16]) {
+    const int ql = threadIdx.x & 7;
+    const uint32_t s = (8u - (R & 7u)) & 7u;
+    const uint32_t r8 = R + s;                       // kept bits: 16, 24 or 32
+    const uint32_t pdrop = 1u << (32u - r8);         // x 2^drop: the kept bytes to the top
+    const uint32_t ps = 1u << s;                     // x 2^s: Formula 5's left shift
+    // this lane's 16 codes (4 bytes at a + 1 + 4 ql, any alignment)
+    uint32_t codes;
+    {
+        const uint32_t ca = a + 1u + 4u * (uint32_t)ql;
+        const uint32_t w0 = lds_u32(ca & ~3u), w1 = lds_u32((ca & ~3u) + 4u);
+        codes = __funnelshift_r(w0, w1, 8u * (ca & 3u));
+    }
+    // copy = min(code, req): only req = 2 caps a code (3 -> 2): clear the low bit of every 3
+    {
+        const uint32_t m = r8 == 16u ? 0x55555555u : 0u;
+        codes ^= codes & (codes >> 1) & m;
+    }
+    // c8 = 8 x bytes copied from the previous value (step 2); m8 = 8 x mid-bytes (step 3);
+    // nm = mask of the bytes NOT copied
+    uint32_t m8[16], nm[16];
+#pragma unroll
+    for (int i = 0; i < 16; i++) {
+        const uint32_t c8 = i == 0 ? (codes << 3) & 24u : i == 1 ? (codes << 1) & 24u : (codes >> (2 * i - 3)) & 24u;
+        m8[i] = r8 - c8;
+        nm[i] = 0xFFFFFFFFu >> c8;
+    }
+    uint32_t pre[8];  // bit offset of pair p within the lane's run
+    pre[0] = 0;
+#pragma unroll
+    for (int p = 1; p < 8; p++) pre[p] = pre[p - 1] + m8[2 * p - 2] + m8[2 * p - 1];
+    const uint32_t msum = (pre[7] + m8[14] + m8[15]) >> 3;
+    uint32_t incl = shfl_up_add8<1>(msum);
+    incl = shfl_up_add8<2>(incl);
+    incl = shfl_up_add8<4>(incl);
+    const uint32_t tot = __shfl_sync(0xffffffffu, incl, 7, 8);
+    const bool ok = 33u + tot == z;
+    const uint32_t o = a + 33u + incl - msum;
+    // value i's mid-bytes moved to their place under the copied top bytes
+    uint32_t sw[16];
+#pragma unroll
+    for (int p = 0; p < 8; p++) {
+        uint32_t r[2];
+        run_load_s<2>(o + (pre[p] >> 3), r);
+        sw[2 * p] = r[0] * pdrop;
+        sw[2 * p + 1] = __funnelshift_rc(r[0], r[1], m8[2 * p]) * pdrop;
+    }
+    // lane map c -> (c & M) | D, then its exclusive scan within the quarter
+    uint32_t orm = nm[0];
+#pragma unroll
+    for (int i = 1; i < 16; i++) orm |= nm[i];
+    uint32_t cM = ~orm;
+    uint32_t cD = sw[0] & nm[0];
+#pragma unroll
+    for (int i = 1; i < 16; i++) cD = (cD & ~nm[i]) | (sw[i] & nm[i]);
+#pragma unroll
+    for (int d = 1; d < 8; d <<= 1) {
+        const uint32_t pM = __shfl_up_sync(0xffffffffu, cM, d, 8);
+        const uint32_t pD = __shfl_up_sync(0xffffffffu, cD, d, 8);
+        cD = (pD & cM) | cD;   // lanes below d get their own map back (idempotent)
+        cM = pM & cM;
+    }
+    uint32_t prev = __shfl_up_sync(0xffffffffu, cD, 1, 8);
+    prev = ql == 0 ? 0u : prev;
+#pragma unroll
+    for (int i = 0; i < 16; i++) {
+        const uint32_t w = (prev & ~nm[i]) | (sw[i] & nm[i]);
+        prev = w;
+        out[i] = __fadd_rn(__uint_as_float(w * ps), mu);
+    }
+    return ok;
+}
+
 // decode_full with the payload in global memory
 template <typename T, int VPL, typename Src>
 __device__ inline bool decode_full_g(const Src src, uint32_t z, T mu, T (&out)[VPL]) {
@@ -732,6 +830,7 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
     constexpr int QB = B * W / LY::CB;  // chunks per block
     extern __shared__ __align__(16) uint8_t dsm[];
     __shared__ uint64_t s_w[32];
+    __shared__ uint32_t s_sel[8][32];  // per warp: the selected blocks of a segment, in rank order
     QualAcc qa;
     const T* __restrict__ ref = static_cast<const T*>(p.ref);
     pdl_wait();
@@ -891,7 +990,63 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
         const uint32_t sel = __ballot_sync(0xffffffffu, insg) & rm;
         const uint32_t offl = __shfl_sync(0xffffffffu, z.zincl - z.zl, rank);
         const uint32_t zzl = __shfl_sync(0xffffffffu, z.zl, rank);
-        if constexpr (sizeof(T) == 4 && VPL == 4) {
+        if constexpr (sizeof(T) == 4 && VPL == 4 && SZX_DQUARTER) {
+            // four blocks per iteration, a quarter-warp each (16 values per lane).
+            // Lane r of s_sel holds the index of the r-th selected block.
+            const int q = lane >> 3, ql = lane & 7;
+            const uint32_t wq = threadIdx.x >> 5;
+            if ((sel >> lane) & 1u) s_sel[wq][__popc(sel & ((1u << lane) - 1u))] = (uint32_t)lane;
+            __syncwarp();
+            const uint32_t nsel = __popc(sel);
+            float* yb = reinterpret_cast<float*>(y) + t * TB * B + ql * 16;
+#pragma unroll 1
+            for (uint32_t r0 = 0; r0 < nsel; r0 += 4) {
+                const bool act = r0 + q < nsel;
+                const int jq = (int)s_sel[wq][act ? r0 + q : r0];
+                const uint32_t off = __shfl_sync(0xffffffffu, offl, jq);
+                const uint32_t zz = __shfl_sync(0xffffffffu, zzl, jq);
+                const float mu = __uint_as_float(__shfl_sync(0xffffffffu, (uint32_t)m.mul, jq));
+                const uint32_t aq = sbase + off;
+                const uint32_t R = lds_u8(aq);
+                if (__all_sync(0xffffffffu, R >= 9u && R < 32u)) {
+                    float v[16];
+                    const bool ok = decode_quarter_f32x16(aq, R, zz, mu, v);
+                    if (act) {
+                        if (!ok) {
+                            if (ql == 0) set_corrupt(p.err);
+                        } else {
+                            uint4* qo = reinterpret_cast<uint4*>(yb + jq * B);
+#pragma unroll
+                            for (int c = 0; c < 4; c++) st_out16(qo + c, reinterpret_cast<const uint4*>(v)[c]);
+                            if constexpr (QUAL) {
+                                const uint4* rq = reinterpret_cast<const uint4*>(ref + t * TB * B + jq * B + ql * 16);
+                                qa.add16<T, 4>(rq, reinterpret_cast<const uint4(&)[4]>(v));
+                            }
+                        }
+                    }
+                } else {
+                    // a raw (R = 32) or malformed block among the four: whole-warp generic decoder
+                    const uint32_t nb = nsel - r0 < 4u ? nsel - r0 : 4u;
+                    for (uint32_t k = 0; k < nb; k++) {
+                        const int j = (int)s_sel[wq][r0 + k];
+                        const uint32_t offj = __shfl_sync(0xffffffffu, offl, j);
+                        const uint32_t zj = __shfl_sync(0xffffffffu, zzl, j);
+                        const T muj = TR::from(__shfl_sync(0xffffffffu, m.mul, j));
+                        T v[VPL];
+                        if (!decode_full_g<T, VPL>(SrcS{sbase + offj}, zj, muj, v)) {
+                            if (lane == 0) set_corrupt(p.err);
+                            continue;
+                        }
+#pragma unroll
+                        for (int qq = 0; qq < NV; qq++) st_out(yq + j * QB + qq, reinterpret_cast<const V*>(v)[qq]);
+                        if constexpr (QUAL)
+                            qa.add16<T, NV, V>(reinterpret_cast<const V*>(ref + t * TB * B + lane * VPL) + j * QB,
+                                               reinterpret_cast<const V(&)[NV]>(v));
+                    }
+                }
+            }
+            __syncwarp();  // s_sel is rewritten by the next segment
+        } else if constexpr (sizeof(T) == 4 && VPL == 4) {
             // two blocks per iteration, a half-warp each (the second half idles
             // on the last block of an odd count)
             const int h = lane >> 4, hl = lane & 15;

@@ -100,9 +100,12 @@ __device__ inline uint64_t okey_inv(uint64_t k) { return dkey_inv(k); }
 
 // eb_abs from the global finite range keys (reading R13): REL x (max - min)
 // in double, canonical +0; no finite values -> 0.
-__device__ inline double eb_from_range(int mode, double eb_user, const uint64_t* range_keys) {
+__device__ inline double eb_from_range(int mode, double eb_user, const uint64_t* range_keys,
+                                       const double* eb_abs_in = nullptr) {
     double e;
-    if (mode == 0) {
+    if (eb_abs_in) {  // the caller already holds the (global) absolute bound
+        e = *eb_abs_in;
+    } else if (mode == 0) {
         e = eb_user;
     } else {
         if (!range_keys || range_keys[0] == ~0ull) {

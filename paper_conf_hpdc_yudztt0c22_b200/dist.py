@@ -41,11 +41,11 @@ def shard_elems(n: int, b: int, P: int, p: int) -> tuple[int, int]:
     return e0, max(0, e1 - e0)
 
 
-def allreduce_range_keys(keys: torch.Tensor, group=None) -> torch.Tensor:
+def allreduce_range_keys(keys: torch.Tensor, group=None, force: bool = False) -> torch.Tensor:
     """Element-wise MIN of [key(min), ~key(max)] (uint64 bit patterns held in int64) over ranks."""
     if group is None and not (dist.is_available() and dist.is_initialized()):
         return keys
-    if dist.get_world_size(group) == 1:
+    if dist.get_world_size(group) == 1 and not force:
         return keys
     k = torch.bitwise_xor(keys, torch.full_like(keys, _FLIP))
     dist.all_reduce(k, op=dist.ReduceOp.MIN, group=group)
@@ -102,7 +102,8 @@ class ShardedCompressor:
       -> all-gather of (n_elem, stream bytes) so every rank knows the container offsets.
     """
 
-    def __init__(self, n_local: int, dtype=torch.float32, block_size: int = 128, device="cuda", group=None):
+    def __init__(self, n_local: int, dtype=torch.float32, block_size: int = 128, device="cuda", group=None,
+                 force_collectives: bool = False):
         from . import szx as _szx
         self._szx = _szx
         self.n, self.b, self.group = n_local, block_size, group
@@ -117,18 +118,35 @@ class ShardedCompressor:
         self.rec = torch.zeros(2, dtype=torch.int64, device=device)
         ws = dist.get_world_size(group) if dist.is_available() and dist.is_initialized() else 1
         self.world = ws
+        # run the collectives even on a 1-rank group (the bench's torchrun --nproc-per-node 1 path
+        # exercises the same NCCL calls, captured in the step's CUDA graph, as N > 1)
+        self.collectives = ws > 1 or (force_collectives and dist.is_available() and dist.is_initialized())
         self.records = torch.zeros(ws * 2, dtype=torch.int64, device=device)
 
     def compress(self, x: torch.Tensor, eb: float, mode="rel", stream=None):
+        """Enqueue the shard's compression on `stream` (default: the current stream).
+
+        Every step -- the two C-ABI calls, the key and record copies and both
+        collectives -- is issued on that one stream (torch's collectives run on
+        the current stream's order for NCCL), so the all-reduce reads the local
+        keys after szx_local_range wrote them, the encoder reads the global keys
+        after the all-reduce, and the record all-gather reads the stream length
+        after the encoder wrote it."""
+        if stream is not None and x.is_cuda:
+            with torch.cuda.stream(stream):
+                return self._compress(x, eb, mode)
+        return self._compress(x, eb, mode)
+
+    def _compress(self, x: torch.Tensor, eb: float, mode):
         L = self._szx.lib()
         m = self._szx._mode_code(mode)
-        st = self._szx._stream(stream)
+        st = self._szx._stream(None)
         assert x.is_contiguous() and x.numel() == self.n and x.dtype == self.dtype
         xp = x.data_ptr() if self.n else None
         self._szx._check(L.szx_local_range(xp, self.dt, self.n, self.b, self.keys.data_ptr(), self.ws.data_ptr(),
                                            self.ws.numel(), st), "szx_local_range")
-        if m == self._szx.REL and self.world > 1:
-            self.keys.copy_(allreduce_range_keys(self.keys, self.group))
+        if m == self._szx.REL and self.collectives:
+            self.keys.copy_(allreduce_range_keys(self.keys, self.group, force=True))
         self._szx._check(L.szx_compress_shard_async(xp, self.dt, self.n, m, float(eb),
                                                     ctypes.c_void_p(self.keys.data_ptr()), self.b,
                                                     self.out.data_ptr(), self.cap, self.ws.data_ptr(),
@@ -136,7 +154,7 @@ class ShardedCompressor:
                          "szx_compress_shard_async")
         self.rec[0] = self.n
         self.rec[1:2].copy_(self.total)
-        if self.world > 1:
+        if self.collectives:
             dist.all_gather_into_tensor(self.records, self.rec, group=self.group)
         else:
             self.records.copy_(self.rec)

@@ -71,6 +71,8 @@ def lib() -> ctypes.CDLL:
         "szx_load_host": (i64, [vp, u64, vp, u64, vp]),
         "szx_local_range": (i32, [vp, i32, u64, u32, vp, vp, u64, vp]),
         "szx_compress_shard_async": (i32, [vp, i32, u64, i32, dbl, vp, u32, vp, u64, vp, u64, vp, vp]),
+        "szx_local_minmax": (i32, [vp, i32, u64, vp, vp]),
+        "szx_compress_shard": (i64, [vp, i32, u64, i32, dbl, vp, u32, vp, u64, vp]),
         "szx_timing_enable": (None, [i32]),
         "szx_timing_reset": (None, []),
         "szx_timing_read": (i32, [ctypes.POINTER(ctypes.c_char_p), ctypes.POINTER(dbl),
@@ -94,6 +96,7 @@ EXPORTED = ["szx_compress_bound", "szx_compress_workspace_bytes", "szx_decompres
             "szx_decompress", "szx_decompress_blocks", "szx_decompress_ws", "szx_decompress_async", "szx_compress_host",
             "szx_decompress_host", "szx_decompress_quality", "szx_decompress_quality_async",
             "szx_quality_finish", "szx_dump_host", "szx_load_host", "szx_local_range", "szx_compress_shard_async",
+            "szx_local_minmax", "szx_compress_shard",
             "szx_timing_enable", "szx_timing_reset", "szx_timing_read", "szx_launch_count",
             "szx_debug_set_r_bias", "szx_strerror"]
 
@@ -347,6 +350,34 @@ def decompress_host(s, out=None, stream=None):
                                   _stream(stream))
     _check(r, "szx_decompress_host")
     return out[:n]
+
+
+def local_minmax(x: torch.Tensor, stream=None) -> torch.Tensor:
+    """SURVEY 8(b) szx_local_minmax: (min, max) of the finite values of a CUDA tensor, as a float64
+    device tensor of 2 (no finite value -> (+inf, -inf)); non-blocking."""
+    _require_cuda(x)
+    x = x.contiguous().view(-1)
+    mm = torch.empty(2, dtype=torch.float64, device=x.device)
+    _check(lib().szx_local_minmax(x.data_ptr() if x.numel() else None, _dtype_code(x), x.numel(), mm.data_ptr(),
+                                  _stream(stream)), "szx_local_minmax")
+    return mm
+
+
+def compress_shard(x: torch.Tensor, eb: float, eb_abs: torch.Tensor, mode="rel", block_size: int = 128,
+                   out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """SURVEY 8(b) szx_compress_shard: compress a shard with the absolute bound held on the device
+    (eb_abs: float64 CUDA tensor of 1); blocking, returns the stream (uint8 CUDA tensor)."""
+    _require_cuda(x)
+    x = x.contiguous().view(-1)
+    dt = _dtype_code(x)
+    cap = compress_bound(x.numel(), dt, block_size)
+    if out is None:
+        out = torch.empty(cap, dtype=torch.uint8, device=x.device)
+    assert eb_abs.is_cuda and eb_abs.dtype == torch.float64 and eb_abs.is_contiguous()
+    nb = _check(lib().szx_compress_shard(x.data_ptr() if x.numel() else None, dt, x.numel(), _mode_code(mode),
+                                         float(eb), eb_abs.data_ptr(), block_size, out.data_ptr(), out.numel(),
+                                         _stream(stream)), "szx_compress_shard")
+    return out[:nb]
 
 
 class Codec:

@@ -116,7 +116,7 @@ def run_case(x: torch.Tensor, eb: float, iters: int, flush: torch.Tensor | None,
     nb = n * W
     pk = peak()
     return {"n": n, "dtype": "f32" if W == 4 else "f64", "stream_bytes": S, "cr": nb / S,
-            "nonconst_frac": h.n_nonconst / ((n + 127) // 128), "eb_abs": h.eb_abs, "max_abs_err": err,
+            "nonconst_frac": h.n_nonconst / ((n + b - 1) // b), "eb_abs": h.eb_abs, "max_abs_err": err,
             "compress_ms": cms, "decompress_ms": dms,
             "compress_gbs": nb / cms / 1e6, "decompress_gbs": nb / dms / 1e6,
             "compress_hbm_frac": (2 * nb + S) / cms / 1e6 / pk, "decompress_hbm_frac": (S + nb) / dms / 1e6 / pk,

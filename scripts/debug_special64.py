@@ -3,6 +3,7 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np, torch
 import oracle, synth
 import paper_conf_hpdc_yudztt0c22_b200 as szx
+sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tests"))
 from fig10_decoder import decode as fdec
 x = synth.special_values(123_457, 9).numpy().astype(np.float64)
 ref, tr = oracle.compress(x, 1e-2, oracle.REL, 128, trace=True)

@@ -175,3 +175,31 @@ def test_decompress_blocks_errors():
     with pytest.raises(S.SZxError) as e:
         szx.decompress_blocks(bad, 0, 5)
     assert e.value.code == -3  # ECORRUPT
+
+
+@pytest.mark.parametrize("dt", [np.float32, np.float64])
+def test_minmax_and_compress_shard_double_forms(dt):
+    """SURVEY 8(b)'s double-valued boundary: szx_local_minmax of every shard, the MIN/MAX combine an
+    all-reduce would do, eb_abs = REL x (max - min) in double (footnote 1), then the
+    blocking szx_compress_shard with that device-held bound: each shard stream is byte-identical to
+    the oracle's shard stream with the oracle's global bound."""
+    x = synth.special_values(200_003, 17, dtype=torch.float32 if dt == np.float32 else torch.float64).cuda()
+    n, P, b, rel = x.numel(), 3, 128, 1e-3
+    parts = [sdist.shard_elems(n, b, P, p) for p in range(P)]
+    mms = [szx.local_minmax(x[f:f + c]) for f, c in parts]
+    gmin = torch.stack([m[0] for m in mms]).min()
+    gmax = torch.stack([m[1] for m in mms]).max()
+    xn = x.cpu().numpy()
+    fin = xn[np.isfinite(xn)]
+    assert gmin.item() == float(fin.min()) and gmax.item() == float(fin.max())
+    e_ref = oracle.eb_abs(xn, rel, oracle.REL)
+    eb_abs = (rel * (gmax - gmin)).reshape(1).contiguous()
+    assert eb_abs.item() == e_ref
+    for f, c in parts:
+        got = szx.compress_shard(x[f:f + c], rel, eb_abs, "rel", b).cpu().numpy()
+        ref = oracle.compress_shard(xn[f:f + c], rel, e_ref, oracle.REL, b)
+        assert got.tobytes() == ref.tobytes(), (f, c)
+    # a shard without finite values
+    nan = torch.full((300,), float("nan"), dtype=x.dtype, device="cuda")
+    mm = szx.local_minmax(nan).cpu().tolist()
+    assert mm[0] == float("inf") and mm[1] == float("-inf")
