@@ -1,6 +1,7 @@
 """Build libszx_b200.so in-tree with nvcc for sm_100a (no JIT, no torch extension)."""
 from __future__ import annotations
 
+import glob
 import os
 import subprocess
 
@@ -9,9 +10,8 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libszx_b200.so")
 SOURCES = [os.path.join(CSRC, "szx_api.cu")]
-DEPS = SOURCES + [os.path.join(CSRC, f) for f in ("szx_device.cuh", "szx_compress.cuh",
-                                                   "szx_decompress.cuh")] + [
-    os.path.join(ROOT, "include", "szx.h")]
+DEPS = sorted(glob.glob(os.path.join(CSRC, "*.cu")) + glob.glob(os.path.join(CSRC, "*.cuh"))) + [
+    os.path.join(ROOT, "include", "szx.h"), os.path.abspath(__file__)]
 
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 # IEEE round-to-nearest everywhere: no FMA contraction, no flush-to-zero, exact div/sqrt.

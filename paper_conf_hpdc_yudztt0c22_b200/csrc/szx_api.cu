@@ -9,12 +9,14 @@
 #include <cmath>
 #include <cstring>
 #include <map>
+#include <type_traits>
 #include <mutex>
 #include <vector>
 
 #include "../../include/szx.h"
 #include "szx_compress.cuh"
 #include "szx_decompress.cuh"
+#include "szx_encode.cuh"
 
 using namespace szx;
 
@@ -172,7 +174,7 @@ uint64_t cdiv(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
 
 // ------------------------------------------------------------ compress layout
 struct CLayout {
-    uint64_t nB, nW, nTB, nTC;
+    uint64_t nB, nW, nTB, nTC, nTE;
     uint64_t off_keys, off_zero, zero_bytes, off_scal, off_stats, off_nclist, off_nckeys, off_ncR, off_gbase,
         off_codes, codes_bytes, total;
 };
@@ -184,7 +186,8 @@ CLayout clayout(uint64_t n, int W, uint32_t b) {
     L.nTC = cdiv(cdiv(L.nB, kWriteTile), 256);  // k_zscan CTAs (look-back status words)
     L.off_keys = 0;
     L.off_zero = 16;
-    L.zero_bytes = al16(16 + 8 * L.nTB + 8 * L.nTC);
+    L.nTE = cdiv(L.nB, 4 * SZX_ENW) + 1;  // k_encode_f32 tiles (look-back status words)
+    L.zero_bytes = al16(16 + 8 * L.nTB + 8 * L.nTC + 16 * L.nTE);
     L.off_scal = L.off_zero + L.zero_bytes;
     L.off_stats = L.off_scal + 32;
     L.off_nclist = al16(L.off_stats + 2ull * W * L.nB);
@@ -209,6 +212,8 @@ Plan make_plan(const CLayout& L, uint8_t* ws, uint64_t n, szx_dtype_t dt, szx_eb
     p.ctr = reinterpret_cast<uint32_t*>(ws + L.off_zero);
     p.status_b = reinterpret_cast<uint64_t*>(ws + L.off_zero + 16);
     p.status_c = p.status_b + L.nTB;
+    p.status_e = p.status_c + L.nTC;
+    p.prefix_e = p.status_e + L.nTE;
     p.eb_abs = reinterpret_cast<double*>(ws + L.off_scal);
     p.nnc = reinterpret_cast<uint64_t*>(ws + L.off_scal + 8);
     p.total = reinterpret_cast<uint64_t*>(ws + L.off_scal + 16);
@@ -273,7 +278,7 @@ KernelSetup& kernel_setup() { static KernelSetup k; return k; }
 // Blocks of `k` per SM at 256 threads with `smem` dynamic bytes on the current
 // device (attributes set on first use per device); `dflt` if the query fails.
 template <typename K>
-int kernel_occupancy(K k, size_t smem, int dflt) {
+int kernel_occupancy(K k, size_t smem, int dflt, int threads = 256) {
     int dev = 0;
     if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return dflt; }
     KernelSetup& S = kernel_setup();
@@ -284,7 +289,7 @@ int kernel_occupancy(K k, size_t smem, int dflt) {
     carve(k);
     if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     int occ = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, 256, smem) != cudaSuccess || occ <= 0) {
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, threads, smem) != cudaSuccess || occ <= 0) {
         cudaGetLastError();
         occ = dflt;
     }
@@ -315,6 +320,23 @@ void enqueue_encode(const void* d_in, const Plan& p, const CLayout& L, uint8_t* 
     kernel_occupancy(k_classify<T>, 0, 1);
     kernel_occupancy(k_zscan<Traits<T>::W>, 0, 1);
     launch("k_classify", s, [&] { launch_pdl(k_classify<T>, dim3((unsigned)L.nTB), dim3(256), 0, s, p, out); });
+#ifndef SZX_FUSED
+#define SZX_FUSED 1   // float32 b = 128: the fused single-pass encoder (szx_encode.cuh)
+#endif
+    if constexpr (std::is_same<T, float>::value && VPL == 4) {
+        if (SZX_FUSED) {
+            using EC = EncCfg<SZX_ENW, SZX_ENS>;
+            auto kern = k_encode_f32<SZX_ENW, SZX_ENS>;
+            const int occ_e = kernel_occupancy(kern, EC::SMEM, 1, EC::NT);
+            const uint64_t egrid = std::max<uint64_t>(
+                1, std::min<uint64_t>(cdiv(L.nB, EC::TILE), (uint64_t)sm_count() * occ_e));
+            launch("k_encode", s, [&] {
+                launch_coop(kern, dim3((unsigned)egrid), dim3(EC::NT), EC::SMEM, s, static_cast<const float*>(d_in),
+                            p, out);
+            });
+            return;
+        }
+    }
     const int occ = kernel_occupancy(k_enc_size<T, VPL>, SizeCfg<T, VPL>::SMEM, 2);
     uint64_t grid = cdiv(L.nB, 8);
     const uint64_t cap = (uint64_t)sm_count() * occ;

@@ -45,7 +45,9 @@ struct Plan {
     const double* eb_in;       // non-null: the absolute bound, given (szx_compress_shard)
     uint32_t* ctr;             // [4] tile tickets, init 0
     uint64_t* status_b;        // classify look-back, init 0
-    uint64_t* status_c;        // encode look-back, init 0
+    uint64_t* status_c;        // offset-scan look-back, init 0
+    uint64_t* status_e;        // fused encoder: tile sizes (one word per tile), init 0
+    uint64_t* prefix_e;        // fused encoder: tile payload offsets from the scanner, init 0
     void* stats;               // 2 keys per block (min, max)
     uint32_t* nclist;          // ids of the nonconstant blocks, in block order
     void* ncmu;                // their mu (bits), same order

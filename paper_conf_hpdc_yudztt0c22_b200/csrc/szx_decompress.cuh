@@ -169,6 +169,9 @@ __device__ inline uint64_t cta_scan256(uint64_t v, uint64_t* agg, uint64_t* s_w 
 #ifndef SZX_STCS
 #define SZX_STCS 1
 #endif
+#ifndef SZX_DNR
+#define SZX_DNR 1        // float32 b = 128 half-warp decoder: non-raw fast form
+#endif
 #ifndef SZX_DQUARTER
 #define SZX_DQUARTER 0   // float32 b = 128: quarter-warp (1) or half-warp (0) block decoder
 #endif
@@ -576,6 +579,68 @@ __device__ __forceinline__ bool decode_half_f32x8(uint32_t a, uint32_t z, float 
         const uint32_t w = (prev & ~nm[i]) | (sw[i] & nm[i]);
         prev = w;
         out[i] = raw ? __uint_as_float(w) : __fadd_rn(__uint_as_float(w << s), mu);
+    }
+    return ok;
+}
+
+// decode_half_f32x8 for non-raw blocks (9 <= R < 32, read by the caller):
+// the shifts by the block constants drop and s are multiplications by powers
+// of two (FMA pipe), the code cap min(code, req) is applied once per lane to
+// the packed codes, and there is no raw select per value.
+__device__ __forceinline__ bool decode_half_f32x8_nr(uint32_t a, uint32_t R, uint32_t z, float mu,
+                                                     float (&out)[8]) {
+    const int sl = threadIdx.x & 15;
+    const uint32_t s = (8u - (R & 7u)) & 7u;
+    const uint32_t r8 = R + s;                     // kept bits: 16, 24 or 32
+    const uint32_t pdrop = 1u << (32u - r8);
+    const uint32_t ps = 1u << s;
+    uint32_t codes = lds_u8(a + 1 + 2 * sl) | (lds_u8(a + 2 + 2 * sl) << 8);
+    codes ^= codes & (codes >> 1) & (r8 == 16u ? 0x5555u : 0u);  // req = 2: code 3 copies 2 bytes
+    uint32_t m8[8], nm[8];
+#pragma unroll
+    for (int i = 0; i < 8; i++) {
+        const uint32_t c8 = i == 0 ? (codes << 3) & 24u : i == 1 ? (codes << 1) & 24u : (codes >> (2 * i - 3)) & 24u;
+        m8[i] = r8 - c8;
+        nm[i] = 0xFFFFFFFFu >> c8;
+    }
+    const uint32_t b01 = m8[0] + m8[1], b23 = m8[2] + m8[3], b45 = m8[4] + m8[5];
+    const uint32_t msum = (b01 + b23 + b45 + m8[6] + m8[7]) >> 3;
+    uint32_t incl = shfl_up_add16<1>(msum);
+    incl = shfl_up_add16<2>(incl);
+    incl = shfl_up_add16<4>(incl);
+    incl = shfl_up_add16<8>(incl);
+    const uint32_t tot = __shfl_sync(0xffffffffu, incl, 15, 16);
+    const bool ok = 33u + tot == z;
+    const uint32_t o = a + 33u + incl - msum;
+    uint32_t r[4][2];
+    run_load_s<2>(o, r[0]);
+    run_load_s<2>(o + (b01 >> 3), r[1]);
+    run_load_s<2>(o + ((b01 + b23) >> 3), r[2]);
+    run_load_s<2>(o + ((b01 + b23 + b45) >> 3), r[3]);
+    uint32_t sw[8];
+#pragma unroll
+    for (int q = 0; q < 4; q++) {
+        sw[2 * q] = r[q][0] * pdrop;
+        sw[2 * q + 1] = __funnelshift_rc(r[q][0], r[q][1], m8[2 * q]) * pdrop;
+    }
+    uint32_t cM = ~(nm[0] | nm[1] | nm[2] | nm[3] | nm[4] | nm[5] | nm[6] | nm[7]);
+    uint32_t cD = sw[0] & nm[0];
+#pragma unroll
+    for (int i = 1; i < 8; i++) cD = (cD & ~nm[i]) | (sw[i] & nm[i]);
+#pragma unroll
+    for (int d = 1; d < 16; d <<= 1) {
+        const uint32_t pM = __shfl_up_sync(0xffffffffu, cM, d, 16);
+        const uint32_t pD = __shfl_up_sync(0xffffffffu, cD, d, 16);
+        cD = (pD & cM) | cD;
+        cM = pM & cM;
+    }
+    uint32_t prev = __shfl_up_sync(0xffffffffu, cD, 1, 16);
+    prev = sl == 0 ? 0u : prev;
+#pragma unroll
+    for (int i = 0; i < 8; i++) {
+        const uint32_t w = (prev & ~nm[i]) | (sw[i] & nm[i]);
+        prev = w;
+        out[i] = __fadd_rn(__uint_as_float(w * ps), mu);
     }
     return ok;
 }
@@ -1063,7 +1128,14 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
                 const uint32_t zz = __shfl_sync(0xffffffffu, zzl, jh);
                 const float mu = __uint_as_float(__shfl_sync(0xffffffffu, (uint32_t)m.mul, jh));
                 float v[8];
+#if SZX_DNR
+                const uint32_t Rh = lds_u8(sbase + off);
+                const bool ok = __all_sync(0xffffffffu, Rh >= 9u && Rh < 32u)
+                                    ? decode_half_f32x8_nr(sbase + off, Rh, zz, mu, v)
+                                    : decode_half_f32x8(sbase + off, zz, mu, v);
+#else
                 const bool ok = decode_half_f32x8(sbase + off, zz, mu, v);
+#endif
                 if (h == 0 || two) {
                     if (!ok) {
                         if (hl == 0) set_corrupt(p.err);

@@ -1,0 +1,535 @@
+// szx_encode.cuh -- fused single-pass encoder for float32, b = 128 (sm_100a).
+//
+//   k_encode_f32 (K2+K3+K4 in one pass over the nonconstant blocks)
+//
+// One read of the nonconstant blocks' values, one write of the payload: per
+// tile of 32 nonconstant blocks (the compacted list of k_classify, in block
+// order) a 256-thread CTA
+//   (1) stages the tile's 32 x 512 B with cp.async (prefetched one tile ahead,
+//       16-byte chunks swizzled so the quarter-warp reads are bank-conflict
+//       free);
+//   (2) encodes every block with a quarter-warp (8 lanes x 16 values): v_i =
+//       d_i - mu (Alg. 1 l.10), Formula 5's shift folded into the lead-byte
+//       count, 2-bit codes min(3, identical leading bytes) against the previous
+//       value (Sec. 6.1 steps 1-4; u_{-1} = 0, reading R6), mid-byte
+//       counts, z_k = 1 + 32 + sum m_i;
+//   (3) scans the tile's z_k (warp 0) and publishes the tile's payload bytes for
+//       the decoupled look-back (the device-wide exclusive scan of block sizes,
+//       P:L2350-2377; 256 predecessors per round trip), warp 0 resolving it
+//       while the other warps pack;
+//   (4) packs [R][codes][mid-bytes] of every block into a zeroed shared-memory
+//       tile with OR reductions (reading R7/R8);
+//   (5) resolves the tile's payload offset and copies the tile out with
+//       16-byte stores, realigned to the output.
+// The R2 guard runs where k_classify could not prove it away (whole-warp
+// check, DESIGN.md s.3); raw blocks (R = 32) and the partial last block take a
+// whole-warp generic path.  Byte-identical to the three-pass encoder and the
+// oracle.
+#pragma once
+
+#include "szx_compress.cuh"
+
+namespace szx {
+
+constexpr int kEncMaxZ = 1 + 32 + 4 * 128;                // float32 b = 128: raw block
+#ifndef SZX_EMINB
+#define SZX_EMINB 5   // encoder CTAs per SM (register budget)
+#endif
+#ifndef SZX_ENW
+#define SZX_ENW 4     // compute warps per encoder CTA (tile = 4 x warps nonconstant blocks)
+#endif
+#ifndef SZX_ENS
+#define SZX_ENS 3     // staging slots per encoder CTA (tiles in flight)
+#endif
+
+// 16-byte chunk c (0..31) of a staged block sits at swz16(c): lane ql of a
+// quarter reads chunks 4 ql .. 4 ql + 3, and the 8 lanes of one LDS.128 phase
+// then hit 8 distinct 16-byte bank groups
+__device__ __forceinline__ uint32_t swz16(uint32_t c) { return (c & ~7u) | ((c ^ (c >> 2)) & 7u); }
+
+// Decoupled look-back with a 256-entry window (8 status words per lane): the
+// exclusive prefix of `agg` over tiles [0, tile).  Tile `tile` must already
+// have published its aggregate (lb_publish).  All 32 lanes of one warp.
+__device__ inline void lb_publish(uint64_t* status, uint64_t tile, uint64_t agg) {
+    st_relaxed(&status[tile], (tile == 0 ? kFlagIncl : kFlagAgg) | agg);
+}
+__device__ inline uint64_t lb_resolve(uint64_t* status, uint64_t tile, uint64_t agg) {
+    constexpr int K = 8;  // status words per lane: a 256-tile window per round trip
+    if (tile == 0) return 0;
+    const int lane = threadIdx.x & 31;
+    uint64_t excl = 0;
+    int64_t base = (int64_t)tile - 1;
+    while (true) {
+        uint64_t st[K];
+#pragma unroll
+        for (int k = 0; k < K; k++) {
+            const int64_t idx = base - K * lane - k;
+            st[k] = idx >= 0 ? ld_relaxed(&status[idx]) : (kFlagIncl | 0);
+        }
+        int kf = K;      // nearest inclusive entry of this lane
+        int kv = K;      // nearest unpublished entry of this lane
+#pragma unroll
+        for (int k = K - 1; k >= 0; k--) {
+            if ((st[k] >> 62) == 2) kf = k;
+            if ((st[k] >> 62) == 0) kv = k;
+        }
+        const uint32_t pm = __ballot_sync(0xffffffffu, kf < K);
+        const int fl = pm ? __ffs(pm) - 1 : 32;            // lane holding the nearest inclusive
+        const int kfl = __shfl_sync(0xffffffffu, kf, fl & 31);
+        // every entry before the nearest inclusive one must be published
+        const bool need_ok = lane < fl ? kv == K : (lane == fl ? kv > kfl : true);
+        if (!__all_sync(0xffffffffu, need_ok)) {
+            // a predecessor has not published yet: one lane polls the nearest such entry
+            // (cheap on L2) before the window is read again
+            const uint32_t um = __ballot_sync(0xffffffffu, kv < K);
+            const int ul = __ffs(um) - 1;
+            const int kvl = __shfl_sync(0xffffffffu, kv, ul);
+            if (lane == 0) {
+                const uint64_t* w = &status[base - K * ul - kvl];
+                uint32_t ns = 64;
+                while (ld_relaxed(w) == 0) {
+                    __nanosleep(ns);
+                    ns = ns < 1024 ? 2 * ns : ns;
+                }
+            }
+            __syncwarp();
+            continue;
+        }
+        uint64_t v = 0;
+#pragma unroll
+        for (int k = 0; k < K; k++) {
+            const bool take = lane < fl || (lane == fl && k <= kfl);
+            v += take ? (st[k] & kValueMask) : 0;
+        }
+        excl += warp_sum64(v);
+        if (pm) break;
+        base -= 32 * K;
+    }
+    if (lane == 0) st_relaxed(&status[tile], kFlagIncl | (excl + agg));
+    return excl;
+}
+
+// Forward scanner of tile sizes (one warp for the whole grid): walks the
+// status array in tile order, 512 tiles per round trip, and writes every
+// tile's exclusive payload offset to prefix[t] (flag bit 63) as soon as the
+// tile and all its predecessors have published their sizes.  Tiles never wait
+// on each other; only a tile's copy-out waits for its own prefix.  The last
+// step completes the stream header (payload bytes) and the total.
+__device__ inline void tile_scanner(const uint64_t* status, uint64_t* prefix, uint64_t ntiles, uint8_t* out,
+                                    uint64_t* total, uint64_t off_pl) {
+#ifndef SZX_ESK
+#define SZX_ESK 8
+#endif
+    constexpr int K = SZX_ESK;     // tiles per lane per window
+    constexpr int WIN = 32 * K;
+    const int lane = threadIdx.x & 31;
+    auto load = [&](uint64_t b, uint64_t (&v)[K]) {
+#pragma unroll
+        for (int k = 0; k < K; k++) {
+            const uint64_t t = b + (uint64_t)(K * lane + k);
+            v[k] = t < ntiles ? ld_relaxed(&status[t]) : 0;
+        }
+    };
+    uint64_t base = 0, run = 0;
+    uint32_t ns = 32;
+    uint64_t va[K], vb[K];
+    load(0, va);
+    while (base < ntiles) {
+        // the next window is read while this one is scanned (it is re-read if this one is short)
+        load(base + WIN, vb);
+        int first_bad = K;
+#pragma unroll
+        for (int k = K - 1; k >= 0; k--)
+            if (va[k] == 0) first_bad = k;
+        const uint32_t gap = __ballot_sync(0xffffffffu, first_bad < K);
+        const int gl = gap ? __ffs(gap) - 1 : 32;
+        const int gk = __shfl_sync(0xffffffffu, first_bad, gl & 31);
+        const int nready = gl == 32 ? WIN : K * gl + gk;
+        if (nready == 0) {  // the next tile has not published: back off and re-read
+            __nanosleep(ns);
+            ns = ns < 512 ? 2 * ns : ns;
+            load(base, va);
+            continue;
+        }
+        ns = 32;
+        uint64_t loc = 0, pre[K];
+#pragma unroll
+        for (int k = 0; k < K; k++) {
+            pre[k] = loc;
+            loc += K * lane + k < nready ? (va[k] & kValueMask) : 0;
+        }
+        uint64_t incl = loc;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint64_t tt = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl += tt;
+        }
+        const uint64_t lex = run + incl - loc;
+#pragma unroll
+        for (int k = 0; k < K; k++)
+            if (K * lane + k < nready) st_relaxed(&prefix[base + K * lane + k], (1ull << 63) | (lex + pre[k]));
+        run += __shfl_sync(0xffffffffu, incl, 31);
+        base += (uint64_t)nready;
+        if (nready == WIN) {
+#pragma unroll
+            for (int k = 0; k < K; k++) va[k] = vb[k];
+        } else {
+            load(base, va);
+        }
+    }
+    if (lane == 0) {
+        reinterpret_cast<uint64_t*>(out)[6] = run;  // header: payload bytes
+        *total = off_pl + run;
+    }
+}
+
+// ---- quarter-warp block encoder (full float32 block, 9 <= R < 32)
+struct QEnc {
+    uint32_t v[16];     // normalised words bits(d_i - mu)
+    uint32_t codes;     // 2-bit lead codes of the lane's 16 values, LSB-first
+    uint32_t msum;      // mid-bytes of the lane
+};
+
+// Formula 5: s = (8 - R % 8) % 8, req = (R + s) / 8.  The lead-byte count of
+// the shifted words u = v >> s is min(3, (clz(v_i ^ v_{i-1}) + s) / 8): a
+// logical shift adds s identical leading zeros to both words; OR-ing 0xFF << s
+// into the XOR caps the count at 3.
+__device__ __forceinline__ void quarter_encode_f32(const float (&x)[16], float mu, uint32_t R, QEnc& e,
+                                                   uint32_t (&m8)[16]) {
+    const int ql = threadIdx.x & 7;
+    const uint32_t s = (8u - (R & 7u)) & 7u;
+    const uint32_t req = (R + s) >> 3;
+    const uint32_t cap = 0xFFu << s;
+#pragma unroll
+    for (int i = 0; i < 16; i++) e.v[i] = __float_as_uint(__fsub_rn(x[i], mu));
+    uint32_t prev = __shfl_up_sync(0xffffffffu, e.v[15], 1, 8);
+    prev = ql == 0 ? 0u : prev;
+    uint32_t codes = 0, msum = 0;
+#pragma unroll
+    for (int i = 0; i < 16; i++) {
+        const uint32_t L = ((uint32_t)__clz((e.v[i] ^ prev) | cap) + s) >> 3;
+        prev = e.v[i];
+        codes |= L << (2 * i);
+        const uint32_t m = req - umin(L, req);
+        m8[i] = 8u * m;
+        msum += m;
+    }
+    e.codes = codes;
+    e.msum = msum;
+}
+
+// Pack the quarter's block at shared byte address dst: [R][32 code bytes][mid-bytes];
+// mexcl = this lane's exclusive mid-byte offset within the block.
+__device__ __forceinline__ void quarter_pack_f32(const QEnc& e, const uint32_t (&m8)[16], uint32_t R,
+                                                 uint32_t mexcl, uint32_t dst) {
+    const int ql = threadIdx.x & 7;
+    if (ql == 0) red_or_s(dst & ~3u, R << (8u * (dst & 3u)));
+    {   // this lane's 4 code bytes at dst + 1 + 4 ql (two words at most)
+        const uint32_t a = dst + 1u + 4u * (uint32_t)ql, sh = 8u * (a & 3u);
+        red_or_s(a & ~3u, e.codes << sh);
+        red_or_nz((a & ~3u) + 4u, __funnelshift_l(e.codes, 0u, sh));
+    }
+    const uint32_t rs = 32u - R;     // v >> rs = the R kept bits (u >> drop)
+    uint32_t a = dst + 33u + mexcl;
+#pragma unroll
+    for (int h = 0; h < 8; h++) {
+        const uint32_t n0 = m8[2 * h], n1 = m8[2 * h + 1];
+        // the mid-bytes: the low m_i bytes of the kept bits (bytes [W-req, W-L) of u)
+        const uint32_t c0 = (e.v[2 * h] >> rs) & ~__funnelshift_lc(0u, 0xFFFFFFFFu, n0);
+        const uint32_t c1 = (e.v[2 * h + 1] >> rs) & ~__funnelshift_lc(0u, 0xFFFFFFFFu, n1);
+        const uint32_t lo = c0 | __funnelshift_lc(0u, c1, n0);
+        const uint32_t hi = __funnelshift_lc(c1, 0u, n0);
+        const uint32_t sh = 8u * (a & 3u), wa = a & ~3u;
+        red_or_s(wa, lo << sh);
+        red_or_s(wa + 4u, __funnelshift_l(lo, hi, sh));
+        red_or_nz(wa + 8u, __funnelshift_l(hi, 0u, sh));
+        a += (n0 + n1) >> 3;
+    }
+}
+
+template <int O>
+__device__ __forceinline__ uint32_t shfl_up_add8e(uint32_t v) {
+    asm volatile(
+        "{\n\t.reg .u32 t;\n\t.reg .pred p;\n\t"
+        "shfl.sync.up.b32 t|p, %0, %1, 0x1800, -1;\n\t"
+        "@p add.u32 %0, %0, t;\n\t}"
+        : "+r"(v)
+        : "n"(O));
+    return v;
+}
+
+// Copy the packed tile [0, T) of the staging area (shared address stg, 16-byte
+// aligned, 16 readable bytes before it) to global g0, with 16-byte stores; the
+// two boundary chunks are shared with the neighbouring tiles and written word-
+// or byte-wise.  The realignment is tile-uniform: staging byte s lands at
+// global g0 + s, so output chunk ch (at A + 16 ch, A = g0 & ~15) holds staging
+// bytes [16 ch - d, +16), d = g0 & 15.
+template <int NT>
+__device__ __forceinline__ void copy_out_tile(uint32_t stg, uint8_t* g0, uint32_t T) {
+    const uintptr_t a0 = reinterpret_cast<uintptr_t>(g0), A = a0 & ~uintptr_t(15), E = a0 + T;
+    const uint32_t d = (uint32_t)(a0 - A);
+    const uint32_t nch = (uint32_t)((E - A + 15) >> 4);
+    const uint32_t wsh = (16u - d) >> 2, sh = 8u * ((16u - d) & 3u);  // window start (in words) within chunks ch-1, ch
+    for (uint32_t ch = threadIdx.x; ch < nch; ch += NT) {
+        const uint4 p0 = lds_u128(stg + 16u * ch - 16u), p1 = lds_u128(stg + 16u * ch);
+        const uint32_t w8[8] = {p0.x, p0.y, p0.z, p0.w, p1.x, p1.y, p1.z, p1.w};
+        uint32_t w[5];
+        // w[k] = w8[wsh + k] (wsh in 0..4; the branch is uniform over the tile)
+        switch (wsh) {
+            case 0: w[0] = w8[0]; w[1] = w8[1]; w[2] = w8[2]; w[3] = w8[3]; w[4] = w8[4]; break;
+            case 1: w[0] = w8[1]; w[1] = w8[2]; w[2] = w8[3]; w[3] = w8[4]; w[4] = w8[5]; break;
+            case 2: w[0] = w8[2]; w[1] = w8[3]; w[2] = w8[4]; w[3] = w8[5]; w[4] = w8[6]; break;
+            case 3: w[0] = w8[3]; w[1] = w8[4]; w[2] = w8[5]; w[3] = w8[6]; w[4] = w8[7]; break;
+            default: w[0] = w8[4]; w[1] = w8[5]; w[2] = w8[6]; w[3] = w8[7]; w[4] = 0u; break;
+        }
+        uint4 v;
+        v.x = __funnelshift_r(w[0], w[1], sh);
+        v.y = __funnelshift_r(w[1], w[2], sh);
+        v.z = __funnelshift_r(w[2], w[3], sh);
+        v.w = __funnelshift_r(w[3], w[4], sh);
+        const uintptr_t a = A + 16 * (uintptr_t)ch;
+        if (a >= a0 && a + 16 <= E) {
+            *reinterpret_cast<uint4*>(a) = v;
+        } else {
+            const uint32_t vw[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+            for (int qq = 0; qq < 4; qq++) {
+                const uintptr_t aw = a + 4 * qq;
+                if (aw >= a0 && aw + 4 <= E) {
+                    *reinterpret_cast<uint32_t*>(aw) = vw[qq];
+                } else if (aw + 4 > a0 && aw < E) {
+                    for (int c = 0; c < 4; c++)
+                        if (aw + c >= a0 && aw + c < E) *reinterpret_cast<uint8_t*>(aw + c) = (uint8_t)(vw[qq] >> (8 * c));
+                }
+            }
+        }
+    }
+}
+
+template <int NW, int NS>
+struct EncCfg {
+    static constexpr int NTC = 32 * NW;               // compute threads
+    static constexpr int NT = NTC + 32;               // + the look-back warp
+    static constexpr int TILE = 4 * NW;               // nonconstant blocks per tile (a quarter-warp each)
+    static constexpr int IN = TILE * 512;             // the tile's values
+    static constexpr int STG = (TILE * kEncMaxZ + 64 + 15) / 16 * 16;
+    static constexpr int SMEM = 2 * IN + NS * (16 + STG); // 2 x input | NS x (16-byte pad | staging slot)
+};
+
+__device__ __forceinline__ void bar_compute(int nthreads) {
+    asm volatile("bar.sync 1, %0;" ::"r"(nthreads) : "memory");
+}
+__device__ __forceinline__ uint32_t ld_vol_s(const uint32_t* p) { return *reinterpret_cast<const volatile uint32_t*>(p); }
+
+// Software-pipelined fused encoder.  NW compute warps work on tile k (ticket,
+// staging, encode, z-scan, publish the tile size, pack into staging slot
+// k % NS) and copy tile k out NS - 1 tiles later, once the grid's tile scanner
+// (the extra warp of CTA 0) has produced its payload offset; the scan latency
+// and the jitter of other tiles' publishes overlap with the next tiles' work.
+// Tiles are handed out in ticket order and publish without waiting, so the
+// scanner always advances; the grid is co-resident (cooperative launch), so
+// the scanner's CTA runs.
+template <int NW, int NS>
+__global__ void __launch_bounds__(32 * NW + 32, SZX_EMINB) k_encode_f32(const float* __restrict__ x, Plan p,
+                                                                       uint8_t* __restrict__ out) {
+    using C = EncCfg<NW, NS>;
+    constexpr int B = 128;
+    extern __shared__ __align__(16) uint8_t esm[];
+    __shared__ uint32_t s_z[C::TILE], s_off[C::TILE];
+    __shared__ uint64_t s_cur;
+    __shared__ uint64_t s_tile[NS], s_excl[NS];
+    __shared__ uint32_t s_T[NS];
+    pdl_wait();
+    pdl_trigger();
+    const uint64_t nnc = *p.nnc;
+    const double eb = *p.eb_abs;
+    const uint64_t ntiles = (nnc + C::TILE - 1) / C::TILE;
+    const uint64_t off_zs = p.off_mu + al16(4 * p.nB);
+    const uint64_t off_pl = off_zs + al16(2 * nnc);
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const uint32_t ib = smem_u32(esm);
+    auto slot_addr = [&](int sl) -> uint32_t { return ib + 2 * C::IN + 16u + (uint32_t)sl * (16u + C::STG); };
+
+    for (uint32_t c = tid; c < NS * (16 + C::STG) / 16; c += C::NT)  // OR reductions assemble tiles in zeroed staging
+        asm volatile("st.shared.v4.u32 [%0], {%1,%1,%1,%1};" ::"r"(ib + 2 * C::IN + 16u * c), "r"(0u) : "memory");
+    __syncthreads();
+
+    if (warp == NW) {
+        // the grid's tile scanner runs in the extra warp of CTA 0; the others leave
+        if (blockIdx.x == 0 && ntiles) tile_scanner(p.status_e, p.prefix_e, ntiles, out, p.total, off_pl);
+        return;
+    }
+
+    // ---------------- compute warps
+    uint16_t* zsize = reinterpret_cast<uint16_t*>(out + off_zs);
+    uint32_t* mus = reinterpret_cast<uint32_t*>(out + p.off_mu);
+    const uint32_t* ncmu = reinterpret_cast<const uint32_t*>(p.ncmu);
+    const uint32_t nBfull = (uint32_t)(p.n / B);       // block ids fit 32 bits (kMaxN / 32)
+    const uint32_t nnc32 = (uint32_t)nnc;
+    const int q = lane >> 3, ql = lane & 7;
+    const int j = warp * 4 + q;  // this quarter's block within the tile
+    // copy out tile kk (its offset produced by the scanner), then zero its slot
+    auto retire = [&](uint32_t kk) {
+        const int sl = (int)(kk % NS);
+        if (tid == 0) {
+            uint64_t v;
+            uint32_t ns = 32;
+            while (!((v = ld_relaxed(&p.prefix_e[s_tile[sl]])) >> 63)) {
+                __nanosleep(ns);
+                ns = ns < 256 ? 2 * ns : ns;
+            }
+            s_excl[sl] = v & ~(1ull << 63);
+        }
+        bar_compute(C::NTC);
+        const uint32_t T = s_T[sl];
+        copy_out_tile<C::NTC>(slot_addr(sl), out + off_pl + s_excl[sl], T);
+        bar_compute(C::NTC);
+        for (uint32_t c = tid; c < (T + 15u) / 16u + 2u; c += C::NTC)
+            asm volatile("st.shared.v4.u32 [%0], {%1,%1,%1,%1};" ::"r"(slot_addr(sl) + 16u * c), "r"(0u) : "memory");
+    };
+    // metadata of this warp's 4 blocks of tile t (lanes 0-3); the values are staged by
+    // the warp itself into its part of input buffer b (lane l: chunks (l & 7) + 8 kk of block l >> 3)
+    struct Meta { uint32_t mk, mu, rec; };
+    auto load_meta = [&](uint32_t t) -> Meta {
+        Meta m{0xFFFFFFFFu, 0u, 9u | 0x80u};
+        const uint32_t nc0 = t * (uint32_t)C::TILE + 4u * (uint32_t)warp;
+        if (t < ntiles && lane < 4 && nc0 + lane < nnc32) {
+            m.mk = p.nclist[nc0 + lane];
+            m.mu = ncmu[nc0 + lane];
+            m.rec = p.ncR[nc0 + lane];
+        }
+        return m;
+    };
+    auto stage = [&](const Meta& m, int b) {
+        const uint32_t bk = __shfl_sync(0xffffffffu, m.mk, lane >> 3);
+        if (bk < nBfull) {
+            const uint32_t dst = ib + (uint32_t)b * C::IN + (uint32_t)warp * 2048u + (uint32_t)q * 512u;
+#pragma unroll
+            for (int kk = 0; kk < 4; kk++) {
+                const uint32_t c = (uint32_t)(ql + 8 * kk);
+                cp_async16(dst + 16u * swz16(c), x + (uint64_t)bk * B + 4u * c);
+            }
+        }
+        cp_async_commit();
+    };
+    if (tid == 0) s_cur = atomicAdd(&p.ctr[3], 1u);
+    bar_compute(C::NTC);
+    uint32_t cur = (uint32_t)s_cur;
+    Meta mc = load_meta(cur);
+    if (cur < ntiles) stage(mc, 0);
+    uint32_t k = 0;
+    for (;; k++) {
+        const int slot = (int)(k % NS);
+        const uint32_t stg = slot_addr(slot);
+        const int buf = (int)(k & 1);
+        bar_compute(C::NTC);  // (A) s_cur consumed; the slot is free and zeroed
+        if (cur >= ntiles) break;
+        if (tid == 0) s_cur = atomicAdd(&p.ctr[3], 1u);  // the next tile (prefetched below)
+        const uint32_t wib = ib + (uint32_t)buf * C::IN + (uint32_t)warp * 2048u;  // this warp's 4 staged blocks
+        const uint32_t mk = __shfl_sync(0xffffffffu, mc.mk, q);
+        const float mu = __uint_as_float(__shfl_sync(0xffffffffu, mc.mu, q));
+        const uint32_t rec = __shfl_sync(0xffffffffu, mc.rec, q);
+        const bool valid = cur * (uint32_t)C::TILE + 4u * (uint32_t)warp + (uint32_t)q < nnc32;
+        uint32_t R = rec & 0x7Fu;
+        const bool full = mk < nBfull;
+        cp_async_wait<0>();
+        __syncwarp();  // the warp's own blocks are staged
+        {   // R2 guard where classify could not prove it away: whole warp, one block at a time
+            const bool ng = valid && full && !(rec & 0x80u) && R < 32u;
+            uint32_t gm = __ballot_sync(0xffffffffu, ng && ql == 0);
+            while (gm) {
+                const int gl = __ffs(gm) - 1;
+                gm &= gm - 1;
+                float xw[4];
+                reinterpret_cast<uint4*>(xw)[0] = lds_u128(wib + (uint32_t)(gl >> 3) * 512u + 16u * swz16((uint32_t)lane));
+                const float gmu = __shfl_sync(0xffffffffu, mu, gl);
+                const int gR = (int)__shfl_sync(0xffffffffu, R, gl);
+                const int fR = guard_R<float, 4>(xw, 4, gmu, gR, eb);
+                if ((lane >> 3) == (gl >> 3)) R = (uint32_t)fR;
+            }
+        }
+        const bool fast = !__any_sync(0xffffffffu, valid && (!full || R >= 32u));
+        QEnc e;
+        uint32_t m8[16];
+        uint32_t mexcl = 0;
+        auto generic = [&](bool pack) {
+            // whole-warp encoder, one block at a time (raw blocks, the partial last block)
+            for (int kq = 0; kq < 4; kq++) {
+                const int bj = warp * 4 + kq;
+                const bool bv = __shfl_sync(0xffffffffu, valid, 8 * kq);
+                const uint32_t bk = __shfl_sync(0xffffffffu, mk, 8 * kq);
+                const float bmu = __shfl_sync(0xffffffffu, mu, 8 * kq);
+                const int bR = (int)__shfl_sync(0xffffffffu, R, 8 * kq);
+                if (!bv) {
+                    if (!pack && lane == 0) s_z[bj] = 0u;
+                    continue;
+                }
+                float xw[4];
+                uint32_t uu[4];
+                LaneCode lc;
+                int cnt = 4, len = B;
+                if (bk < nBfull) {
+                    reinterpret_cast<uint4*>(xw)[0] = lds_u128(wib + (uint32_t)kq * 512u + 16u * swz16((uint32_t)lane));
+                } else {
+                    cnt = load_lane<float, 4>(x, p.n, bk, lane, xw);
+                    len = (int)(p.n - (uint64_t)bk * B);
+                }
+                encode_known_R<float, 4>(xw, cnt, len, bR >= 32 ? 0.0f : bmu, bR, uu, lc);
+                if (!pack) {
+                    if (lane == 0) s_z[bj] = lc.z;
+                } else {
+                    pack_red<float, 4>(uu, lc, cnt, len, stg + s_off[bj]);
+                    if (lane == 0 && bR >= 32) mus[bk] = 0u;  // raw: mu = +0 (R15)
+                }
+            }
+        };
+        if (fast) {
+            float xv[16];
+#pragma unroll
+            for (int kq = 0; kq < 4; kq++)
+                reinterpret_cast<uint4*>(xv)[kq] = lds_u128(wib + (uint32_t)q * 512u + 16u * swz16(4u * ql + kq));
+            quarter_encode_f32(xv, mu, valid ? R : 9u, e, m8);
+            uint32_t incl = shfl_up_add8e<1>(e.msum);
+            incl = shfl_up_add8e<2>(incl);
+            incl = shfl_up_add8e<4>(incl);
+            mexcl = incl - e.msum;
+            const uint32_t tot = __shfl_sync(0xffffffffu, incl, 7, 8);
+            if (ql == 0) s_z[j] = valid ? 33u + tot : 0u;
+        } else {
+            generic(false);
+        }
+        bar_compute(C::NTC);  // (C) every block's z_k; the next ticket
+        const uint32_t nxt = (uint32_t)s_cur;
+        const Meta mn = load_meta(nxt);
+        if (warp == 0) {
+            const uint32_t zl = lane < C::TILE ? s_z[lane] : 0u;
+            const uint32_t incl = warp_incl_scan(zl);
+            if (lane < C::TILE) s_off[lane] = incl - zl;
+            const uint32_t T = __shfl_sync(0xffffffffu, incl, 31);
+            const uint32_t ncl = cur * (uint32_t)C::TILE + (uint32_t)lane;
+            if (lane < C::TILE && ncl < nnc32) zsize[ncl] = (uint16_t)zl;
+            if (lane == 0) {
+                st_relaxed(&p.status_e[cur], kFlagAgg | T);  // the tile's size, for the scanner
+                s_T[slot] = T;
+                s_tile[slot] = cur;
+            }
+        }
+        bar_compute(C::NTC);  // (D) in-tile offsets
+        if (fast) {
+            if (valid) quarter_pack_f32(e, m8, R, mexcl, stg + s_off[j]);
+        } else {
+            generic(true);
+        }
+        // the next tile's values: its metadata arrived during the scan / pack
+        if (nxt < ntiles) stage(mn, buf ^ 1);
+        bar_compute(C::NTC);  // (E) packed
+        if (k + 1 >= NS) retire(k + 1 - NS);
+        cur = nxt;
+        mc = mn;
+    }
+    // drain: the tiles still in their slots, in order
+    const uint32_t k0 = k + 1 >= NS ? k + 1 - NS : 0;
+    for (uint32_t kk = k0; kk < k; kk++) retire(kk);
+}
+
+}  // namespace szx
