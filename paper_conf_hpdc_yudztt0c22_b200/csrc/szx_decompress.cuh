@@ -592,8 +592,9 @@ __device__ __forceinline__ bool decode_half_f32x8_nr(uint32_t a, uint32_t R, uin
     const int sl = threadIdx.x & 15;
     const uint32_t s = (8u - (R & 7u)) & 7u;
     const uint32_t r8 = R + s;                     // kept bits: 16, 24 or 32
-    const uint32_t pdrop = 1u << (32u - r8);
-    const uint32_t ps = 1u << s;
+    // opaque powers of two: the shifts by drop and s become IMADs (FMA pipe), not SHFs
+    const uint32_t pdrop = launder(1u << (32u - r8));
+    const uint32_t ps = launder(1u << s);
     uint32_t codes = lds_u8(a + 1 + 2 * sl) | (lds_u8(a + 2 + 2 * sl) << 8);
     codes ^= codes & (codes >> 1) & (r8 == 16u ? 0x5555u : 0u);  // req = 2: code 3 copies 2 bytes
     uint32_t m8[8], nm[8];
@@ -670,8 +671,8 @@ __device__ __forceinline__ bool decode_quarter_f32x16(uint32_t a, uint32_t R, ui
     const int ql = threadIdx.x & 7;
     const uint32_t s = (8u - (R & 7u)) & 7u;
     const uint32_t r8 = R + s;                       // kept bits: 16, 24 or 32
-    const uint32_t pdrop = 1u << (32u - r8);         // x 2^drop: the kept bytes to the top
-    const uint32_t ps = 1u << s;                     // x 2^s: Formula 5's left shift
+    const uint32_t pdrop = launder(1u << (32u - r8));  // x 2^drop: the kept bytes to the top (IMAD)
+    const uint32_t ps = launder(1u << s);              // x 2^s: Formula 5's left shift (IMAD)
     // this lane's 16 codes (4 bytes at a + 1 + 4 ql, any alignment)
     uint32_t codes;
     {

@@ -201,7 +201,8 @@ __device__ inline uint32_t lds_u32(uint32_t a) {
 // Run of bytes starting at an arbitrary shared address, realigned into NW words.
 template <int NW>
 __device__ inline void run_load_s(uint32_t a, uint32_t (&r)[NW]) {
-    const uint32_t base = a & ~3u, sh = 8 * (a & 3u);
+    // __funnelshift_r wraps its amount mod 32, so 8 a selects the byte offset a & 3
+    const uint32_t base = a & ~3u, sh = 8 * a;
     uint32_t lo = lds_u32(base);
 #pragma unroll
     for (int q = 0; q < NW; q++) {

@@ -381,11 +381,8 @@ __global__ void __launch_bounds__(32 * NW + 32, SZX_EMINB) k_encode_f32(const fl
             s_excl[sl] = v & ~(1ull << 63);
         }
         bar_compute(C::NTC);
-        const uint32_t T = s_T[sl];
-        copy_out_tile<C::NTC>(slot_addr(sl), out + off_pl + s_excl[sl], T);
-        bar_compute(C::NTC);
-        for (uint32_t c = tid; c < (T + 15u) / 16u + 2u; c += C::NTC)
-            asm volatile("st.shared.v4.u32 [%0], {%1,%1,%1,%1};" ::"r"(slot_addr(sl) + 16u * c), "r"(0u) : "memory");
+        copy_out_tile<C::NTC>(slot_addr(sl), out + off_pl + s_excl[sl], s_T[sl]);
+        // (the slot is zeroed when it is reused, NS - 1 tiles later)
     };
     // metadata of this warp's 4 blocks of tile t (lanes 0-3); the values are staged by
     // the warp itself into its part of input buffer b (lane l: chunks (l & 7) + 8 kk of block l >> 3)
@@ -422,8 +419,13 @@ __global__ void __launch_bounds__(32 * NW + 32, SZX_EMINB) k_encode_f32(const fl
         const int slot = (int)(k % NS);
         const uint32_t stg = slot_addr(slot);
         const int buf = (int)(k & 1);
-        bar_compute(C::NTC);  // (A) s_cur consumed; the slot is free and zeroed
+        bar_compute(C::NTC);  // (A) s_cur consumed; the slot's previous tile is copied out
         if (cur >= ntiles) break;
+        if (k >= NS) {  // zero what the slot's previous tile used (ordered before the pack by (C))
+            const uint32_t To = s_T[slot];
+            for (uint32_t c = tid; c < (To + 15u) / 16u + 2u; c += C::NTC)
+                asm volatile("st.shared.v4.u32 [%0], {%1,%1,%1,%1};" ::"r"(stg + 16u * c), "r"(0u) : "memory");
+        }
         if (tid == 0) s_cur = atomicAdd(&p.ctr[3], 1u);  // the next tile (prefetched below)
         const uint32_t wib = ib + (uint32_t)buf * C::IN + (uint32_t)warp * 2048u;  // this warp's 4 staged blocks
         const uint32_t mk = __shfl_sync(0xffffffffu, mc.mk, q);
@@ -501,29 +503,31 @@ __global__ void __launch_bounds__(32 * NW + 32, SZX_EMINB) k_encode_f32(const fl
         bar_compute(C::NTC);  // (C) every block's z_k; the next ticket
         const uint32_t nxt = (uint32_t)s_cur;
         const Meta mn = load_meta(nxt);
-        if (warp == 0) {
+        {   // in-tile offsets of the blocks (every warp scans the tile's z_k itself)
             const uint32_t zl = lane < C::TILE ? s_z[lane] : 0u;
             const uint32_t incl = warp_incl_scan(zl);
-            if (lane < C::TILE) s_off[lane] = incl - zl;
+            const uint32_t zoff = __shfl_sync(0xffffffffu, incl - zl, j);
             const uint32_t T = __shfl_sync(0xffffffffu, incl, 31);
-            const uint32_t ncl = cur * (uint32_t)C::TILE + (uint32_t)lane;
-            if (lane < C::TILE && ncl < nnc32) zsize[ncl] = (uint16_t)zl;
-            if (lane == 0) {
-                st_relaxed(&p.status_e[cur], kFlagAgg | T);  // the tile's size, for the scanner
+            if (warp == 0) {
+                const uint32_t ncl = cur * (uint32_t)C::TILE + (uint32_t)lane;
+                if (lane < C::TILE && ncl < nnc32) zsize[ncl] = (uint16_t)zl;
+                if (lane == 0) st_relaxed(&p.status_e[cur], kFlagAgg | T);  // the tile's size, for the scanner
+            }
+            if (fast) {
+                if (valid) quarter_pack_f32(e, m8, R, mexcl, stg + zoff);
+            } else {
+                if (lane < C::TILE) s_off[lane] = incl - zl;  // (same values in every warp)
+                __syncwarp();
+                generic(true);
+            }
+            if (tid == 0) {
                 s_T[slot] = T;
                 s_tile[slot] = cur;
             }
         }
-        bar_compute(C::NTC);  // (D) in-tile offsets
-        if (fast) {
-            if (valid) quarter_pack_f32(e, m8, R, mexcl, stg + s_off[j]);
-        } else {
-            generic(true);
-        }
         // the next tile's values: its metadata arrived during the scan / pack
         if (nxt < ntiles) stage(mn, buf ^ 1);
-        bar_compute(C::NTC);  // (E) packed
-        if (k + 1 >= NS) retire(k + 1 - NS);
+        if (k + 1 >= NS) retire(k + 1 - NS);  // (its barrier also orders this pack before the next zeroing)
         cur = nxt;
         mc = mn;
     }

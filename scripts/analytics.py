@@ -1,6 +1,7 @@
 """SURVEY 8(f) row 1 analytics on the synthetic fields (oracle side, CPU):
 Formula 6 shift overhead (Solution C vs A/B; the Fig. 6
-analogue) and Formula 7 PSNR / max error per field, at the
+analogue) and Formula 7 PSNR / max error per field and block size (8 and 16
+are oracle-only points of the Fig. 8 block-size study), at the
 small shapes the oracle finishes in seconds.  Writes one JSON line per
 (field, eb, b) to stdout."""
 import json
@@ -29,7 +30,7 @@ FIELDS = {
 for name, gen in FIELDS.items():
     x = np.ascontiguousarray(gen()).reshape(-1)
     for eb in (1e-2, 1e-3, 1e-4):
-        for b in (32, 64, 128, 256):
+        for b in (8, 16, 32, 64, 128, 256):
             s = oracle.compress(x, eb, oracle.REL, b)
             y = oracle.decompress(s)
             q = oracle.quality(x, y)
