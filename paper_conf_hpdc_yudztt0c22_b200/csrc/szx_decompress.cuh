@@ -308,16 +308,24 @@ __device__ inline uint32_t ldg_u32(const void* p) { return *reinterpret_cast<con
 // run of bytes at an arbitrary address, realigned; aligned words that start at
 // or past `lim` (one past the last valid byte) read as 0.  An aligned word
 // holding at least one stream byte never leaves the (>=16-B aligned) buffer.
+// the aligned word at w, with the bytes at or past lim read as 0 (never loaded:
+// the caller's buffer may end, or be uninitialised, right after the stream)
+__device__ inline uint32_t ldg_u32_lim(uintptr_t w, uintptr_t lim) {
+    if (w + 4 <= lim) return ldg_u32(reinterpret_cast<const void*>(w));
+    uint32_t v = 0;
+    for (uintptr_t c = w; c < lim; c++) v |= ldg_u8(reinterpret_cast<const uint8_t*>(c)) << (8 * (uint32_t)(c - w));
+    return v;
+}
 template <int NW>
 __device__ inline void run_load(const uint8_t* p, uintptr_t lim4, uint32_t (&r)[NW]) {
     const uintptr_t a = reinterpret_cast<uintptr_t>(p);
     const uintptr_t base = a & ~uintptr_t(3);
     const uint32_t sh = 8 * (uint32_t)(a & 3);
-    uint32_t lo = base < lim4 ? ldg_u32(reinterpret_cast<const void*>(base)) : 0u;
+    uint32_t lo = ldg_u32_lim(base, lim4);
 #pragma unroll
     for (int q = 0; q < NW; q++) {
         const uintptr_t aq = base + 4 * (q + 1);
-        const uint32_t hi = aq < lim4 ? ldg_u32(reinterpret_cast<const void*>(aq)) : 0u;
+        const uint32_t hi = ldg_u32_lim(aq, lim4);
         r[q] = __funnelshift_r(lo, hi, sh);
         lo = hi;
     }

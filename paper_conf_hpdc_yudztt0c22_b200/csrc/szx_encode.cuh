@@ -335,7 +335,7 @@ __global__ void __launch_bounds__(32 * NW + 32, SZX_EMINB) k_encode_f32(const fl
     using C = EncCfg<NW, NS>;
     constexpr int B = 128;
     extern __shared__ __align__(16) uint8_t esm[];
-    __shared__ uint32_t s_z[C::TILE], s_off[C::TILE];
+    __shared__ uint32_t s_z[C::TILE];
     __shared__ uint64_t s_cur;
     __shared__ uint64_t s_tile[NS], s_excl[NS];
     __shared__ uint32_t s_T[NS];
@@ -454,6 +454,8 @@ __global__ void __launch_bounds__(32 * NW + 32, SZX_EMINB) k_encode_f32(const fl
         QEnc e;
         uint32_t m8[16];
         uint32_t mexcl = 0;
+        uint32_t zex = 0;  // lane b < TILE: in-tile payload offset of block b
+        uint32_t rfin = 0;  // generic path: the final R of block kq in byte kq (after the R2 guard)
         auto generic = [&](bool pack) {
             // whole-warp encoder, one block at a time (raw blocks, the partial last block)
             for (int kq = 0; kq < 4; kq++) {
@@ -461,7 +463,8 @@ __global__ void __launch_bounds__(32 * NW + 32, SZX_EMINB) k_encode_f32(const fl
                 const bool bv = __shfl_sync(0xffffffffu, valid, 8 * kq);
                 const uint32_t bk = __shfl_sync(0xffffffffu, mk, 8 * kq);
                 const float bmu = __shfl_sync(0xffffffffu, mu, 8 * kq);
-                const int bR = (int)__shfl_sync(0xffffffffu, R, 8 * kq);
+                const uint32_t brec = __shfl_sync(0xffffffffu, rec, 8 * kq);
+                int bR = pack ? (int)((rfin >> (8 * kq)) & 0xFFu) : (int)__shfl_sync(0xffffffffu, R, 8 * kq);
                 if (!bv) {
                     if (!pack && lane == 0) s_z[bj] = 0u;
                     continue;
@@ -476,11 +479,18 @@ __global__ void __launch_bounds__(32 * NW + 32, SZX_EMINB) k_encode_f32(const fl
                     cnt = load_lane<float, 4>(x, p.n, bk, lane, xw);
                     len = (int)(p.n - (uint64_t)bk * B);
                 }
-                encode_known_R<float, 4>(xw, cnt, len, bR >= 32 ? 0.0f : bmu, bR, uu, lc);
+                if (!pack && bk >= nBfull && bR < 32) {
+                    // the partial last block: the R2 guard / escalation runs here (R2)
+                    encode_block<float, 4>(xw, cnt, len, bmu, bR, (brec & 0x80u) != 0, eb, uu, lc);
+                    bR = lc.R;
+                } else {
+                    encode_known_R<float, 4>(xw, cnt, len, bR >= 32 ? 0.0f : bmu, bR, uu, lc);
+                }
                 if (!pack) {
+                    rfin |= (uint32_t)bR << (8 * kq);
                     if (lane == 0) s_z[bj] = lc.z;
                 } else {
-                    pack_red<float, 4>(uu, lc, cnt, len, stg + s_off[bj]);
+                    pack_red<float, 4>(uu, lc, cnt, len, stg + __shfl_sync(0xffffffffu, zex, bj));
                     if (lane == 0 && bR >= 32) mus[bk] = 0u;  // raw: mu = +0 (R15)
                 }
             }
@@ -513,11 +523,10 @@ __global__ void __launch_bounds__(32 * NW + 32, SZX_EMINB) k_encode_f32(const fl
                 if (lane < C::TILE && ncl < nnc32) zsize[ncl] = (uint16_t)zl;
                 if (lane == 0) st_relaxed(&p.status_e[cur], kFlagAgg | T);  // the tile's size, for the scanner
             }
+            zex = incl - zl;
             if (fast) {
                 if (valid) quarter_pack_f32(e, m8, R, mexcl, stg + zoff);
             } else {
-                if (lane < C::TILE) s_off[lane] = incl - zl;  // (same values in every warp)
-                __syncwarp();
                 generic(true);
             }
             if (tid == 0) {

@@ -15,6 +15,7 @@ codec itself is the C ABI (szx_local_range + szx_compress_shard_async).
 from __future__ import annotations
 
 import ctypes
+import os
 import struct
 
 import torch
@@ -116,6 +117,7 @@ class ShardedCompressor:
         self.keys = torch.empty(2, dtype=torch.int64, device=device)
         self.total = torch.zeros(1, dtype=torch.int64, device=device)
         self.rec = torch.zeros(2, dtype=torch.int64, device=device)
+        self.rec[0] = n_local  # (constant: set once, so the compress sequence has no host-to-device copy)
         ws = dist.get_world_size(group) if dist.is_available() and dist.is_initialized() else 1
         self.world = ws
         # run the collectives even on a 1-rank group (the bench's torchrun --nproc-per-node 1 path
@@ -152,7 +154,6 @@ class ShardedCompressor:
                                                     self.out.data_ptr(), self.cap, self.ws.data_ptr(),
                                                     self.ws.numel(), self.total.data_ptr(), st),
                          "szx_compress_shard_async")
-        self.rec[0] = self.n
         self.rec[1:2].copy_(self.total)
         if self.collectives:
             dist.all_gather_into_tensor(self.records, self.rec, group=self.group)
@@ -215,3 +216,145 @@ def decompress_local(stream: torch.Tensor, n: int, block_size: int, group=None) 
     nB = (n + block_size - 1) // block_size
     b0, b1 = shard_blocks(nB, world, rank)
     return b0 * block_size, _szx.decompress_blocks(stream, b0, b1 - b0)
+
+
+# --------------------------------------------------------------------------- dump / load
+# SURVEY 8(f) row 3 (the paper's data dumping / loading experiment, Fig. 16) on one
+# box: every rank compresses its block-range shard of a global array with the GLOBAL REL bound and
+# writes its stream into ONE SZXC container file at the offset the all-gathered stream sizes give
+# (rank 0 writes the header and shard table); loading reads a rank's shard (or any shard) back.
+# The per-shard codec is pluggable: CudaShardCodec (this library, the product path) or any object
+# with the same three methods (the CPU oracle in the gloo tests).
+
+class CudaShardCodec:
+    """Per-shard codec over the C ABI: szx_local_minmax, szx_compress_shard (device-held global
+    bound) and szx_decompress; streams are copied to pinned host memory in chunks so the D2H
+    copy of chunk i+1 overlaps the file write of chunk i."""
+
+    def __init__(self, device="cuda"):
+        from . import szx as _szx
+        self._szx = _szx
+        self.device = torch.device(device)
+
+    def local_minmax(self, x: torch.Tensor):
+        return self._szx.local_minmax(x).cpu().tolist() if x.numel() else [float("inf"), float("-inf")]
+
+    def compress(self, x: torch.Tensor, eb: float, eb_abs: float, mode: str, block_size: int) -> torch.Tensor:
+        e = torch.tensor([eb_abs], dtype=torch.float64, device=x.device)
+        return self._szx.compress_shard(x, eb, e, mode, block_size)
+
+    def write(self, fd: int, stream: torch.Tensor, offset: int, chunk: int = 64 << 20) -> None:
+        n = stream.numel()
+        if n == 0:
+            return
+        bufs = [torch.empty(min(chunk, n), dtype=torch.uint8, pin_memory=True) for _ in range(2)]
+        evs = [torch.cuda.Event() for _ in range(2)]
+        cs = torch.cuda.Stream(device=stream.device)
+        cs.wait_stream(torch.cuda.current_stream(stream.device))
+        pos, i = 0, 0
+        pend = None
+        while pos < n or pend is not None:
+            if pos < n:
+                m = min(chunk, n - pos)
+                with torch.cuda.stream(cs):
+                    bufs[i % 2][:m].copy_(stream[pos:pos + m], non_blocking=True)
+                    evs[i % 2].record(cs)
+                cur = (i % 2, pos, m)
+                pos += m
+                i += 1
+            else:
+                cur = None
+            if pend is not None:  # write the previous chunk while this one copies
+                j, p0, m0 = pend
+                evs[j].synchronize()
+                os.pwrite(fd, memoryview(bufs[j][:m0].numpy()), offset + p0)
+            pend = cur
+
+    def read(self, fd: int, offset: int, nbytes: int) -> torch.Tensor:
+        host = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+        got = os.preadv(fd, [memoryview(host.numpy())], offset) if nbytes else 0
+        if got != nbytes:
+            raise IOError(f"short read {got} of {nbytes}")
+        return host.to(self.device, non_blocking=True)
+
+    def decompress(self, stream: torch.Tensor) -> torch.Tensor:
+        return self._szx.decompress(stream)
+
+
+def _rel_bound(rel: float, gmin: float, gmax: float) -> float:
+    """REL x (gmax - gmin) in double over the finite values (reading R13); canonical +0."""
+    if not (gmin <= gmax):  # no finite value anywhere
+        return 0.0
+    e = rel * (gmax - gmin)
+    return e if e != 0.0 else 0.0
+
+
+def dump(x_local, eb: float, path: str, mode: str = "rel", block_size: int = 128, codec=None, group=None):
+    """Write this rank's shard into the SZXC container at `path` (all ranks call it collectively;
+    x_local is shard `rank` of `world`, shard_elems layout).  Returns the container bytes."""
+    import numpy as np
+    codec = codec or CudaShardCodec()
+    world = dist.get_world_size(group) if dist.is_available() and dist.is_initialized() else 1
+    rank = dist.get_rank(group) if world > 1 else 0
+    n_local = int(x_local.numel() if hasattr(x_local, "numel") else len(x_local))
+    # (i) the global finite range (REL): MIN of the minima, MAX of the maxima
+    mn, mx = codec.local_minmax(x_local)
+    if world > 1:
+        t = torch.tensor([mn, -mx], dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MIN, group=group)
+        mn, mx = float(t[0]), -float(t[1])
+    eb_abs = _rel_bound(eb, mn, mx) if mode in ("rel", "REL") else float(eb)
+    s = codec.compress(x_local, eb, eb_abs, mode, block_size)
+    nbytes = int(s.numel() if hasattr(s, "numel") else len(s))
+    # (ii) the container offsets: all-gather of (n_elem, stream bytes)
+    rec = torch.tensor([n_local, nbytes], dtype=torch.int64)
+    if world > 1:
+        recs = [torch.zeros(2, dtype=torch.int64) for _ in range(world)]
+        dist.all_gather(recs, rec, group=group)
+    else:
+        recs = [rec]
+    n_elems = [int(r[0]) for r in recs]
+    sizes = [int(r[1]) for r in recs]
+    _, offs, total = container_layout(n_elems, sizes)
+    if rank == 0:
+        fd = os.open(path, os.O_CREAT | os.O_RDWR | os.O_TRUNC, 0o644)
+        os.ftruncate(fd, total)
+        head = container_header(n_elems, sizes)
+        os.pwrite(fd, head, 0)
+        os.close(fd)
+    if world > 1:
+        dist.barrier(group=group)
+    fd = os.open(path, os.O_RDWR)
+    try:
+        if isinstance(s, torch.Tensor) and s.is_cuda:
+            codec.write(fd, s, offs[rank])
+        else:
+            os.pwrite(fd, np.ascontiguousarray(s, np.uint8).tobytes(), offs[rank])
+        os.fsync(fd) if os.environ.get("SZX_DUMP_FSYNC") else None
+    finally:
+        os.close(fd)
+    if world > 1:
+        dist.barrier(group=group)
+    return total
+
+
+def load(path: str, part: int | None = None, codec=None, group=None):
+    """Read shard `part` (default: this rank's) of the SZXC container at `path` and decode it.
+    Returns (first element, values)."""
+    codec = codec or CudaShardCodec()
+    world = dist.get_world_size(group) if dist.is_available() and dist.is_initialized() else 1
+    rank = dist.get_rank(group) if world > 1 else 0
+    p = rank if part is None else part
+    fd = os.open(path, os.O_RDONLY)
+    try:
+        head = os.pread(fd, CONTAINER_HEAD, 0)
+        if head[:4] != b"SZXC":
+            raise ValueError("not an SZXC container")
+        ver, P = struct.unpack_from("<II", head, 4)
+        if ver != 1 or not (0 <= p < P):
+            raise ValueError("bad container header or shard index")
+        first, n_el, off, nb = struct.unpack("<QQQQ", os.pread(fd, CONTAINER_ENTRY, CONTAINER_HEAD + CONTAINER_ENTRY * p))
+        s = codec.read(fd, off, nb)
+    finally:
+        os.close(fd)
+    return first, codec.decompress(s)

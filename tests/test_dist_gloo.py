@@ -124,3 +124,67 @@ def test_container_layout_closed_form():
     assert offs[0] == 32 + 32 * 4
     # container bytes = 32 + 32P + sum_{p<P-1} al16(S_p) + S_{P-1}  (DESIGN.md s.4)
     assert total == 32 + 32 * 4 + sum((s + 15) // 16 * 16 for s in nbytes[:-1]) + nbytes[-1]
+
+
+class _OracleShardCodec:
+    """The CPU oracle as the per-shard codec of dist.dump / dist.load (test infrastructure)."""
+
+    def local_minmax(self, x):
+        f = x[np.isfinite(x)].astype(np.float64)
+        return (float(f.min()), float(f.max())) if f.size else (float("inf"), float("-inf"))
+
+    def compress(self, x, eb, eb_abs, mode, b):
+        return oracle.compress_shard(x, eb, eb_abs, oracle.REL if mode == "rel" else oracle.ABS, b)
+
+    def read(self, fd, off, nb):
+        return np.frombuffer(os.pread(fd, nb, off), np.uint8)
+
+    def decompress(self, s):
+        return oracle.decompress(s)
+
+
+def _dump_worker(rank, world, port, n, b, rel, path, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        x = synth.random_mix(n, 777).numpy()
+        first, cnt = sdist.shard_elems(n, b, world, rank)
+        total = sdist.dump(x[first:first + cnt], rel, path, "rel", b, codec=_OracleShardCodec())
+        f2, y = sdist.load(path, codec=_OracleShardCodec())
+        fo, yo = sdist.load(path, part=world - 1 - rank, codec=_OracleShardCodec())
+        q.put((rank, total, f2, y.tobytes(), fo, yo.tobytes()))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_two_rank_dump_load_container_file(tmp_path):
+    """two ranks dump their shards into one SZXC file (global REL bound by
+    all-reduce, offsets by all-gather); the file is byte-identical to the oracle's 2-shard
+    container, and each rank loads its own and the other rank's shard bit-exactly."""
+    n, b, rel = 70_001, 128, 1e-3
+    path = str(tmp_path / "dump.szxc")
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_dump_worker, args=(r, 2, port, n, b, rel, path, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    try:
+        res = sorted(q.get(timeout=120) for _ in procs)
+    finally:
+        for p in procs:
+            p.join(timeout=30)
+            if p.is_alive():
+                p.kill()
+    assert all(p.exitcode == 0 for p in procs)
+    x = synth.random_mix(n, 777).numpy()
+    ref = oracle.container_compress(x, rel, oracle.REL, b, 2)
+    data = open(path, "rb").read()
+    assert data == ref.tobytes() and all(r[1] == len(data) for r in res)
+    y = oracle.decompress(ref)
+    for rank, _, f2, yb, fo, yob in res:
+        first, cnt = sdist.shard_elems(n, b, 2, rank)
+        assert f2 == first and yb == y[first:first + cnt].tobytes()
+        fo_, co = sdist.shard_elems(n, b, 2, 1 - rank)
+        assert fo == fo_ and yob == y[fo_:fo_ + co].tobytes()

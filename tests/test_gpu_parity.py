@@ -123,6 +123,21 @@ def test_parity_escalation_path():
         szx.set_r_bias(0)
 
 
+@pytest.mark.parametrize("rb,n", [(-3, 50_000), (-2, 50_000), (-3, 50_048), (-3, 128 * 16 * 5 + 77)])
+def test_parity_escalation_in_partial_last_block(rb, n):
+    """The R2 guard / escalation must also run on the partial last block (a large offset makes
+    the per-block proof fail, so every block is checked value by value; Formula 1)."""
+    x = synth.offset_field(n, 7, 3e3).numpy()
+    try:
+        szx.set_r_bias(rb)
+        got = szx.compress(torch.from_numpy(x).cuda(), 1e-4, "rel", 128).cpu().numpy()
+    finally:
+        szx.set_r_bias(0)
+    ref, tr = oracle.compress(x, 1e-4, oracle.REL, 128, trace=True, r_bias=rb)
+    assert tr.escal.sum() > 0
+    assert got.tobytes() == ref.tobytes()
+
+
 def test_corrupt_streams_are_rejected():
     x = synth.random_mix(50_000, 3).numpy()
     s = szx.compress(torch.from_numpy(x).cuda(), 1e-3, "rel", 128)
