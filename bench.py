@@ -35,6 +35,7 @@ sys.path.insert(0, ROOT)
 METRIC = "SZx compress+decompress throughput, N*W / (T_compress + T_decompress)"
 UNIT = "GB/s"
 FIELD_NAMES = {0: "density", 1: "velocity", 2: "temperature"}
+NCU_NAME = {"k_decode": "k_decode_w", "k_encode": "k_encode_f32"}  # library timing label -> kernel name
 FIELD_DESC = {0: "baryon-density-like exp(2.5g)", 1: "velocity-like 1e7 g", 2: "temperature-like 1e4 exp(0.7g)"}
 
 
@@ -505,10 +506,10 @@ def main():
             moved_c = moved_d = None
             if summ:
                 cks = [k for k in kms if k != "k_decode"]
-                vals = [_ncu_kernel(summ, fname, k) for k in cks]
+                vals = [_ncu_kernel(summ, fname, NCU_NAME.get(k, k)) for k in cks]
                 if cks and all(v and v.get("dram_bytes") is not None for v in vals):
                     moved_c = sum(v["dram_bytes"] for v in vals)
-                vd = _ncu_kernel(summ, fname, "k_decode_w") or _ncu_kernel(summ, fname, "k_decode")
+                vd = _ncu_kernel(summ, fname, "k_decode_w")
                 if vd and vd.get("dram_bytes") is not None:
                     moved_d = vd["dram_bytes"]
             rec["compress_dram_frac"] = (moved_c / (comp_ms[i] / 1e3) / 1e9 / peak) if moved_c else None
@@ -517,7 +518,7 @@ def main():
             if kms:
                 dom = max(kms, key=lambda k: kms[k])
                 ach = alg.get(dom, 0) / (kms[dom] / 1e3) / 1e9
-                nv = _ncu_kernel(summ, fname, {"k_decode": "k_decode_w"}.get(dom, dom))
+                nv = _ncu_kernel(summ, fname, NCU_NAME.get(dom, dom))
                 roofs[fname] = {"kernel": dom, "bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s",
                                 "frac": ach / peak, "peak_kind": peak_kind,
                                 "traffic": nv.get("dram_bytes") if nv else None,

@@ -635,7 +635,7 @@ __device__ __forceinline__ bool decode_half_f32x8_nr(uint32_t a, uint32_t R, uin
     uint32_t cM = ~(nm[0] | nm[1] | nm[2] | nm[3] | nm[4] | nm[5] | nm[6] | nm[7]);
     uint32_t cD = sw[0] & nm[0];
 #pragma unroll
-    for (int i = 1; i < 8; i++) cD = (cD & ~nm[i]) | (sw[i] & nm[i]);
+    for (int i = 1; i < 8; i++) cD = bitsel(cD, sw[i], nm[i]);
 #pragma unroll
     for (int d = 1; d < 16; d <<= 1) {
         const uint32_t pM = __shfl_up_sync(0xffffffffu, cM, d, 16);
@@ -647,7 +647,7 @@ __device__ __forceinline__ bool decode_half_f32x8_nr(uint32_t a, uint32_t R, uin
     prev = sl == 0 ? 0u : prev;
 #pragma unroll
     for (int i = 0; i < 8; i++) {
-        const uint32_t w = (prev & ~nm[i]) | (sw[i] & nm[i]);
+        const uint32_t w = bitsel(prev, sw[i], nm[i]);
         prev = w;
         out[i] = __fadd_rn(__uint_as_float(w * ps), mu);
     }
@@ -958,6 +958,7 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
             U mn = 0;
             if (tn < fill_end) { wn = bm[tn]; mn = mus[tn * TB + lane]; }
             V* yq = reinterpret_cast<V*>(y + t * TB * B + lane * VPL);
+            {
 #pragma unroll 2
             for (uint32_t m = ~word & rmask(t); m; m &= m - 1) {
                 const int j = __ffs(m) - 1;
@@ -970,6 +971,7 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
                 if constexpr (QUAL)
                     qa.add16<T, NV, V>(reinterpret_cast<const V*>(ref + t * TB * B + lane * VPL) + j * QB,
                                        reinterpret_cast<const V(&)[NV]>(v));
+            }
             }
             t = tn;
             word = wn;

@@ -161,6 +161,14 @@ __device__ inline uint32_t warp_incl_scan(uint32_t v) {
     return v;
 }
 
+// (c & ~m) | (v & m) in one LOP3 (the compiler otherwise materialises v & m
+// separately when it is reused)
+__device__ __forceinline__ uint32_t bitsel(uint32_t c, uint32_t v, uint32_t m) {
+    uint32_t d;
+    asm("lop3.b32 %0, %1, %2, %3, 0xD8;" : "=r"(d) : "r"(c), "r"(v), "r"(m));
+    return d;
+}
+
 // ---------------------------------------------------------------- PDL
 // Programmatic dependent launch: wait until the preceding kernel in the stream
 // has completed and its memory is visible (no-op when launched without PDL),
