@@ -323,16 +323,17 @@ void enqueue_encode(const void* d_in, const Plan& p, const CLayout& L, uint8_t* 
 #ifndef SZX_FUSED
 #define SZX_FUSED 1   // float32 b = 128: the fused single-pass encoder (szx_encode.cuh)
 #endif
-    if constexpr (std::is_same<T, float>::value && VPL == 4) {
+    if constexpr (VPL == 4) {
         if (SZX_FUSED) {
-            using EC = EncCfg<SZX_ENW, SZX_ENS>;
-            auto kern = k_encode_f32<SZX_ENW, SZX_ENS>;
+            // b = 128: the fused encoder; float64 keeps 2 staging slots (smem)
+            constexpr int NS = sizeof(T) == 4 ? SZX_ENS : 2;
+            using EC = EncCfg<T, SZX_ENW, NS>;
+            auto kern = k_encode_fused<T, SZX_ENW, NS>;
             const int occ_e = kernel_occupancy(kern, EC::SMEM, 1, EC::NT);
             const uint64_t egrid = std::max<uint64_t>(
                 1, std::min<uint64_t>(cdiv(L.nB, EC::TILE), (uint64_t)sm_count() * occ_e));
             launch("k_encode", s, [&] {
-                launch_coop(kern, dim3((unsigned)egrid), dim3(EC::NT), EC::SMEM, s, static_cast<const float*>(d_in),
-                            p, out);
+                launch_coop(kern, dim3((unsigned)egrid), dim3(EC::NT), EC::SMEM, s, static_cast<const T*>(d_in), p, out);
             });
             return;
         }

@@ -169,6 +169,9 @@ __device__ inline uint64_t cta_scan256(uint64_t v, uint64_t* agg, uint64_t* s_w 
 #ifndef SZX_STCS
 #define SZX_STCS 1
 #endif
+#ifndef SZX_DF64HALF
+#define SZX_DF64HALF 1       // float64 b = 128: half-warp block decoder (8 doubles per lane)
+#endif
 #ifndef SZX_DNR
 #define SZX_DNR 1        // float32 b = 128 half-warp decoder: non-raw fast form
 #endif
@@ -654,6 +657,72 @@ __device__ __forceinline__ bool decode_half_f32x8_nr(uint32_t a, uint32_t R, uin
     return ok;
 }
 
+// ---- two float64 blocks of b = 128 per warp: a half-warp per block, 8 doubles
+// per lane (Fig. 10's five steps).  A value copies at most 3 leading bytes, all
+// in the high word, so the lead-byte chains (the map scan) run on 32-bit high
+// words; the low words are the value's own mid-bytes.  Non-raw blocks
+// (12 <= R < 64).
+__device__ __forceinline__ bool decode_half_f64x8_nr(uint32_t a, uint32_t R, uint32_t z, double mu,
+                                                     double (&out)[8]) {
+    const int sl = threadIdx.x & 15;
+    const uint32_t s = (8u - (R & 7u)) & 7u;
+    const uint32_t r8 = R + s;  // kept bits: 16 .. 64
+    const uint32_t drop = 64u - r8;
+    uint32_t codes = lds_u8(a + 1 + 2 * sl) | (lds_u8(a + 2 + 2 * sl) << 8);
+    codes ^= codes & (codes >> 1) & (r8 == 16u ? 0x5555u : 0u);  // req = 2: code 3 copies 2 bytes
+    uint32_t m8[8], nmh[8];
+#pragma unroll
+    for (int i = 0; i < 8; i++) {
+        const uint32_t c8 = ((codes >> (2 * i)) & 3u) << 3;
+        m8[i] = r8 - c8;
+        nmh[i] = 0xFFFFFFFFu >> c8;  // high-word bytes NOT copied from the previous value
+    }
+    uint32_t msum = 0;
+#pragma unroll
+    for (int i = 0; i < 8; i++) msum += m8[i];
+    msum >>= 3;
+    uint32_t incl = shfl_up_add16<1>(msum);
+    incl = shfl_up_add16<2>(incl);
+    incl = shfl_up_add16<4>(incl);
+    incl = shfl_up_add16<8>(incl);
+    const uint32_t tot = __shfl_sync(0xffffffffu, incl, 15, 16);
+    const bool ok = 33u + tot == z;
+    uint32_t off = a + 33u + incl - msum;
+    uint32_t own_lo[8], own_hi[8];
+#pragma unroll
+    for (int i = 0; i < 8; i++) {
+        uint32_t r[2];
+        run_load_s<2>(off, r);
+        uint64_t c = ((uint64_t)r[1] << 32) | r[0];
+        c = m8[i] >= 64u ? c : (c & ((1ull << m8[i]) - 1ull));
+        const uint64_t own = c << drop;  // the mid-bytes under the copied ones
+        own_lo[i] = (uint32_t)own;
+        own_hi[i] = (uint32_t)(own >> 32);
+        off += m8[i] >> 3;
+    }
+    uint32_t cM = ~(nmh[0] | nmh[1] | nmh[2] | nmh[3] | nmh[4] | nmh[5] | nmh[6] | nmh[7]);
+    uint32_t cD = own_hi[0] & nmh[0];
+#pragma unroll
+    for (int i = 1; i < 8; i++) cD = bitsel(cD, own_hi[i], nmh[i]);
+#pragma unroll
+    for (int d = 1; d < 16; d <<= 1) {
+        const uint32_t pM = __shfl_up_sync(0xffffffffu, cM, d, 16);
+        const uint32_t pD = __shfl_up_sync(0xffffffffu, cD, d, 16);
+        cD = (pD & cM) | cD;
+        cM = pM & cM;
+    }
+    uint32_t prev = __shfl_up_sync(0xffffffffu, cD, 1, 16);
+    prev = sl == 0 ? 0u : prev;
+#pragma unroll
+    for (int i = 0; i < 8; i++) {
+        const uint32_t wh = bitsel(prev, own_hi[i], nmh[i]);
+        prev = wh;
+        const uint64_t w = ((uint64_t)wh << 32) | own_lo[i];
+        out[i] = __dadd_rn(__longlong_as_double((long long)(w << s)), mu);
+    }
+    return ok;
+}
+
 // ---- four float32 blocks of b = 128 per warp: a quarter-warp (8 lanes) per
 // block, 16 values per lane.  Fig. 10's five steps as in
 // decode_half_f32x8; the per-lane steps (R and code parsing, the mid-byte
@@ -890,7 +959,7 @@ struct TileMeta {
 };
 
 template <typename T, int VPL, bool QUAL = false>
-__global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint8_t* __restrict__ in, T* __restrict__ y) {
+__global__ void __launch_bounds__(256, (sizeof(T) == 8 && VPL == 4) ? 2 : SZX_DMINB) k_decode_w(DPlan p, const uint8_t* __restrict__ in, T* __restrict__ y) {
     using TR = Traits<T>;
     using U = typename TR::U;
     using C = DecWCfg<T, VPL>;
@@ -1158,6 +1227,58 @@ __global__ void __launch_bounds__(256, SZX_DMINB) k_decode_w(DPlan p, const uint
                             const uint4* rq = reinterpret_cast<const uint4*>(ref + t * TB * B + jh * B + hl * 8);
                             qa.add16<T, 2>(rq, reinterpret_cast<const uint4(&)[2]>(v));
                         }
+                    }
+                }
+            }
+        } else if constexpr (sizeof(T) == 8 && VPL == 4 && SZX_DF64HALF) {
+            // two float64 blocks per iteration, a half-warp each (8 doubles per lane)
+            const int h = lane >> 4, hl = lane & 15;
+            double* yb = reinterpret_cast<double*>(y) + t * TB * B + hl * 8;
+#pragma unroll 1
+            for (uint32_t bits = sel; bits;) {
+                const int j0 = __ffs(bits) - 1;
+                bits &= bits - 1;
+                const bool two = bits != 0;
+                const int j1 = two ? __ffs(bits) - 1 : j0;
+                bits &= bits - 1;
+                const int jh = h ? j1 : j0;
+                const uint32_t off = __shfl_sync(0xffffffffu, offl, jh);
+                const uint32_t zz = __shfl_sync(0xffffffffu, zzl, jh);
+                const double mu = TR::from(__shfl_sync(0xffffffffu, m.mul, jh));
+                const uint32_t Rh = lds_u8(sbase + off);
+                if (__all_sync(0xffffffffu, Rh >= 12u && Rh < 64u)) {
+                    double v[8];
+                    const bool ok = decode_half_f64x8_nr(sbase + off, Rh, zz, mu, v);
+                    if (h == 0 || two) {
+                        if (!ok) {
+                            if (hl == 0) set_corrupt(p.err);
+                        } else {
+                            uint4* qo = reinterpret_cast<uint4*>(yb + jh * B);
+#pragma unroll
+                            for (int c = 0; c < 4; c++) st_out16(qo + c, reinterpret_cast<const uint4*>(v)[c]);
+                            if constexpr (QUAL) {
+                                const uint4* rq = reinterpret_cast<const uint4*>(ref + t * TB * B + jh * B + hl * 8);
+                                qa.add16<T, 4>(rq, reinterpret_cast<const uint4(&)[4]>(v));
+                            }
+                        }
+                    }
+                } else {
+                    // a raw (R = 64) or malformed block in the pair: whole-warp generic decoder
+                    for (int k2 = 0; k2 < (two ? 2 : 1); k2++) {
+                        const int j = k2 ? j1 : j0;
+                        const uint32_t offj = __shfl_sync(0xffffffffu, offl, j);
+                        const uint32_t zj = __shfl_sync(0xffffffffu, zzl, j);
+                        const T muj = TR::from(__shfl_sync(0xffffffffu, m.mul, j));
+                        T v[VPL];
+                        if (!decode_full_g<T, VPL>(SrcS{sbase + offj}, zj, muj, v)) {
+                            if (lane == 0) set_corrupt(p.err);
+                            continue;
+                        }
+#pragma unroll
+                        for (int qq = 0; qq < NV; qq++) st_out(yq + j * QB + qq, reinterpret_cast<const V*>(v)[qq]);
+                        if constexpr (QUAL)
+                            qa.add16<T, NV, V>(reinterpret_cast<const V*>(ref + t * TB * B + lane * VPL) + j * QB,
+                                               reinterpret_cast<const V(&)[NV]>(v));
                     }
                 }
             }

@@ -27,13 +27,17 @@
 // oracle.
 #pragma once
 
+#include <type_traits>
+
 #include "szx_compress.cuh"
 
 namespace szx {
 
-constexpr int kEncMaxZ = 1 + 32 + 4 * 128;                // float32 b = 128: raw block
 #ifndef SZX_EMINB
 #define SZX_EMINB 5   // encoder CTAs per SM (register budget)
+#endif
+#ifndef SZX_ERED3
+#define SZX_ERED3 1
 #endif
 #ifndef SZX_ENW
 #define SZX_ENW 4     // compute warps per encoder CTA (tile = 4 x warps nonconstant blocks)
@@ -46,6 +50,9 @@ constexpr int kEncMaxZ = 1 + 32 + 4 * 128;                // float32 b = 128: ra
 // quarter reads chunks 4 ql .. 4 ql + 3, and the 8 lanes of one LDS.128 phase
 // then hit 8 distinct 16-byte bank groups
 __device__ __forceinline__ uint32_t swz16(uint32_t c) { return (c & ~7u) | ((c ^ (c >> 2)) & 7u); }
+// the same for CPL chunks per quarter lane (4: float32, 8: float64)
+template <int CPL>
+__device__ __forceinline__ uint32_t swzc(uint32_t c) { return (c & ~7u) | ((c ^ (c / CPL)) & 7u); }
 
 // Decoupled look-back with a 256-entry window (8 status words per lane): the
 // exclusive prefix of `agg` over tiles [0, tile).  Tile `tile` must already
@@ -242,8 +249,70 @@ __device__ __forceinline__ void quarter_pack_f32(const QEnc& e, const uint32_t (
         const uint32_t sh = 8u * (a & 3u), wa = a & ~3u;
         red_or_s(wa, lo << sh);
         red_or_s(wa + 4u, __funnelshift_l(lo, hi, sh));
+#if SZX_ERED3
+        red_or_s(wa + 8u, __funnelshift_l(hi, 0u, sh));  // (unconditional: a predicated ATOMS compiles to a branch)
+#else
         red_or_nz(wa + 8u, __funnelshift_l(hi, 0u, sh));
+#endif
         a += (n0 + n1) >> 3;
+    }
+}
+
+// ---- the same for float64 blocks of b = 128 (8 lanes x 16 doubles): the lead
+// count only needs the high words (three identical leading bytes are decided
+// there; a zero high XOR means >= 4 identical bytes, capped at 3 by the OR)
+struct QEnc64 {
+    uint64_t v[16];
+    uint32_t codes;
+    uint32_t msum;
+};
+__device__ __forceinline__ void quarter_encode_f64(const double (&x)[16], double mu, uint32_t R, QEnc64& e,
+                                                   uint32_t (&m8)[16]) {
+    const int ql = threadIdx.x & 7;
+    const uint32_t s = (8u - (R & 7u)) & 7u;
+    const uint32_t req = (R + s) >> 3;  // 2 .. 8
+    const uint32_t cap = 0xFFu << s;
+#pragma unroll
+    for (int i = 0; i < 16; i++) e.v[i] = (uint64_t)__double_as_longlong(__dsub_rn(x[i], mu));
+    uint32_t prevh = __shfl_up_sync(0xffffffffu, (uint32_t)(e.v[15] >> 32), 1, 8);
+    prevh = ql == 0 ? 0u : prevh;
+    uint32_t codes = 0, msum = 0;
+#pragma unroll
+    for (int i = 0; i < 16; i++) {
+        const uint32_t h = (uint32_t)(e.v[i] >> 32);
+        const uint32_t L = ((uint32_t)__clz((h ^ prevh) | cap) + s) >> 3;
+        prevh = h;
+        codes |= L << (2 * i);
+        const uint32_t m = req - umin(L, req);
+        m8[i] = 8u * m;  // 0 .. 64
+        msum += m;
+    }
+    e.codes = codes;
+    e.msum = msum;
+}
+__device__ __forceinline__ void quarter_pack_f64(const QEnc64& e, const uint32_t (&m8)[16], uint32_t R,
+                                                 uint32_t mexcl, uint32_t dst) {
+    const int ql = threadIdx.x & 7;
+    if (ql == 0) red_or_s(dst & ~3u, R << (8u * (dst & 3u)));
+    {
+        const uint32_t a = dst + 1u + 4u * (uint32_t)ql, sh = 8u * (a & 3u);
+        red_or_s(a & ~3u, e.codes << sh);
+        red_or_nz((a & ~3u) + 4u, __funnelshift_l(e.codes, 0u, sh));
+    }
+    const uint32_t rs = 64u - R;  // v >> rs = the R kept bits
+    uint32_t a = dst + 33u + mexcl;
+#pragma unroll
+    for (int i = 0; i < 16; i++) {
+        const uint32_t n = m8[i];
+        // the low m_i bytes of the kept bits, as (lo, hi) words
+        const uint64_t k = e.v[i] >> rs;
+        const uint64_t c = n >= 64u ? k : (k & ((1ull << n) - 1ull));
+        const uint32_t lo = (uint32_t)c, hi = (uint32_t)(c >> 32);
+        const uint32_t sh = 8u * (a & 3u), wa = a & ~3u;
+        red_or_s(wa, lo << sh);
+        red_or_s(wa + 4u, __funnelshift_l(lo, hi, sh));
+        red_or_s(wa + 8u, __funnelshift_l(hi, 0u, sh));
+        a += n >> 3;
     }
 }
 
@@ -306,34 +375,41 @@ __device__ __forceinline__ void copy_out_tile(uint32_t stg, uint8_t* g0, uint32_
     }
 }
 
-template <int NW, int NS>
+template <typename T, int NW, int NS>
 struct EncCfg {
+    static constexpr int W = (int)sizeof(T);
     static constexpr int NTC = 32 * NW;               // compute threads
-    static constexpr int NT = NTC + 32;               // + the look-back warp
+    static constexpr int NT = NTC + 32;               // + the scanner warp
     static constexpr int TILE = 4 * NW;               // nonconstant blocks per tile (a quarter-warp each)
-    static constexpr int IN = TILE * 512;             // the tile's values
-    static constexpr int STG = (TILE * kEncMaxZ + 64 + 15) / 16 * 16;
+    static constexpr int BW = 128 * W;                // bytes per block
+    static constexpr int CPB = BW / 16;               // 16-byte chunks per block
+    static constexpr int CPL = W;                     // chunks per quarter lane (16 values)
+    static constexpr int MAXZ = 1 + 32 + BW;          // raw block payload
+    static constexpr int IN = TILE * BW;              // the tile's values
+    static constexpr int STG = (TILE * MAXZ + 64 + 15) / 16 * 16;
     static constexpr int SMEM = 2 * IN + NS * (16 + STG); // 2 x input | NS x (16-byte pad | staging slot)
 };
 
 __device__ __forceinline__ void bar_compute(int nthreads) {
     asm volatile("bar.sync 1, %0;" ::"r"(nthreads) : "memory");
 }
-__device__ __forceinline__ uint32_t ld_vol_s(const uint32_t* p) { return *reinterpret_cast<const volatile uint32_t*>(p); }
 
-// Software-pipelined fused encoder.  NW compute warps work on tile k (ticket,
-// staging, encode, z-scan, publish the tile size, pack into staging slot
-// k % NS) and copy tile k out NS - 1 tiles later, once the grid's tile scanner
-// (the extra warp of CTA 0) has produced its payload offset; the scan latency
-// and the jitter of other tiles' publishes overlap with the next tiles' work.
-// Tiles are handed out in ticket order and publish without waiting, so the
-// scanner always advances; the grid is co-resident (cooperative launch), so
-// the scanner's CTA runs.
-template <int NW, int NS>
-__global__ void __launch_bounds__(32 * NW + 32, SZX_EMINB) k_encode_f32(const float* __restrict__ x, Plan p,
-                                                                       uint8_t* __restrict__ out) {
-    using C = EncCfg<NW, NS>;
+// Software-pipelined fused encoder (float32 and float64, b = 128).  NW compute
+// warps work on tile k (ticket, staging, encode, z-scan, publish the tile size,
+// pack into staging slot k % NS) and copy tile k out NS - 1 tiles later, once
+// the grid's tile scanner (the extra warp of CTA 0) has produced its payload
+// offset; the scan latency and the jitter of other tiles' publishes overlap
+// with the next tiles' work.  Tiles are handed out in ticket order and publish
+// without waiting, so the scanner always advances; the grid is co-resident
+// (cooperative launch), so the scanner's CTA runs.
+template <typename T, int NW, int NS>
+__global__ void __launch_bounds__(32 * NW + 32, sizeof(T) == 4 ? SZX_EMINB : 3) k_encode_fused(const T* __restrict__ x, Plan p,
+                                                                         uint8_t* __restrict__ out) {
+    using C = EncCfg<T, NW, NS>;
+    using TR = Traits<T>;
+    using U = typename TR::U;
     constexpr int B = 128;
+    constexpr int W = C::W;
     extern __shared__ __align__(16) uint8_t esm[];
     __shared__ uint32_t s_z[C::TILE];
     __shared__ uint64_t s_cur;
@@ -344,7 +420,7 @@ __global__ void __launch_bounds__(32 * NW + 32, SZX_EMINB) k_encode_f32(const fl
     const uint64_t nnc = *p.nnc;
     const double eb = *p.eb_abs;
     const uint64_t ntiles = (nnc + C::TILE - 1) / C::TILE;
-    const uint64_t off_zs = p.off_mu + al16(4 * p.nB);
+    const uint64_t off_zs = p.off_mu + al16((uint64_t)W * p.nB);
     const uint64_t off_pl = off_zs + al16(2 * nnc);
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const uint32_t ib = smem_u32(esm);
@@ -362,13 +438,13 @@ __global__ void __launch_bounds__(32 * NW + 32, SZX_EMINB) k_encode_f32(const fl
 
     // ---------------- compute warps
     uint16_t* zsize = reinterpret_cast<uint16_t*>(out + off_zs);
-    uint32_t* mus = reinterpret_cast<uint32_t*>(out + p.off_mu);
-    const uint32_t* ncmu = reinterpret_cast<const uint32_t*>(p.ncmu);
+    U* mus = reinterpret_cast<U*>(out + p.off_mu);
+    const U* ncmu = reinterpret_cast<const U*>(p.ncmu);
     const uint32_t nBfull = (uint32_t)(p.n / B);       // block ids fit 32 bits (kMaxN / 32)
     const uint32_t nnc32 = (uint32_t)nnc;
     const int q = lane >> 3, ql = lane & 7;
     const int j = warp * 4 + q;  // this quarter's block within the tile
-    // copy out tile kk (its offset produced by the scanner), then zero its slot
+    // copy out tile kk (its offset produced by the scanner)
     auto retire = [&](uint32_t kk) {
         const int sl = (int)(kk % NS);
         if (tid == 0) {
@@ -386,9 +462,9 @@ __global__ void __launch_bounds__(32 * NW + 32, SZX_EMINB) k_encode_f32(const fl
     };
     // metadata of this warp's 4 blocks of tile t (lanes 0-3); the values are staged by
     // the warp itself into its part of input buffer b (lane l: chunks (l & 7) + 8 kk of block l >> 3)
-    struct Meta { uint32_t mk, mu, rec; };
+    struct Meta { uint32_t mk; U mu; uint32_t rec; };
     auto load_meta = [&](uint32_t t) -> Meta {
-        Meta m{0xFFFFFFFFu, 0u, 9u | 0x80u};
+        Meta m{0xFFFFFFFFu, U(0), 9u | 0x80u};
         const uint32_t nc0 = t * (uint32_t)C::TILE + 4u * (uint32_t)warp;
         if (t < ntiles && lane < 4 && nc0 + lane < nnc32) {
             m.mk = p.nclist[nc0 + lane];
@@ -400,14 +476,21 @@ __global__ void __launch_bounds__(32 * NW + 32, SZX_EMINB) k_encode_f32(const fl
     auto stage = [&](const Meta& m, int b) {
         const uint32_t bk = __shfl_sync(0xffffffffu, m.mk, lane >> 3);
         if (bk < nBfull) {
-            const uint32_t dst = ib + (uint32_t)b * C::IN + (uint32_t)warp * 2048u + (uint32_t)q * 512u;
+            const uint32_t dst = ib + (uint32_t)b * C::IN + (uint32_t)warp * 4u * C::BW + (uint32_t)q * C::BW;
 #pragma unroll
-            for (int kk = 0; kk < 4; kk++) {
+            for (int kk = 0; kk < C::CPB / 8; kk++) {
                 const uint32_t c = (uint32_t)(ql + 8 * kk);
-                cp_async16(dst + 16u * swz16(c), x + (uint64_t)bk * B + 4u * c);
+                cp_async16(dst + 16u * swzc<C::CPL>(c), x + (uint64_t)bk * B + (16 / W) * c);
             }
         }
         cp_async_commit();
+    };
+    // the warp-layout values of block kq (lane l: values 4 l .. 4 l + 3) from the staged tile
+    auto warp_vals = [&](uint32_t wib, int kq, T (&xw)[4]) {
+#pragma unroll
+        for (int h = 0; h < 4 * W / 16; h++)
+            reinterpret_cast<uint4*>(xw)[h] =
+                lds_u128(wib + (uint32_t)kq * C::BW + 16u * swzc<C::CPL>((uint32_t)(lane * (4 * W / 16) + h)));
     };
     if (tid == 0) s_cur = atomicAdd(&p.ctr[3], 1u);
     bar_compute(C::NTC);
@@ -427,9 +510,9 @@ __global__ void __launch_bounds__(32 * NW + 32, SZX_EMINB) k_encode_f32(const fl
                 asm volatile("st.shared.v4.u32 [%0], {%1,%1,%1,%1};" ::"r"(stg + 16u * c), "r"(0u) : "memory");
         }
         if (tid == 0) s_cur = atomicAdd(&p.ctr[3], 1u);  // the next tile (prefetched below)
-        const uint32_t wib = ib + (uint32_t)buf * C::IN + (uint32_t)warp * 2048u;  // this warp's 4 staged blocks
+        const uint32_t wib = ib + (uint32_t)buf * C::IN + (uint32_t)warp * 4u * C::BW;  // this warp's 4 staged blocks
         const uint32_t mk = __shfl_sync(0xffffffffu, mc.mk, q);
-        const float mu = __uint_as_float(__shfl_sync(0xffffffffu, mc.mu, q));
+        const T mu = TR::from(__shfl_sync(0xffffffffu, mc.mu, q));
         const uint32_t rec = __shfl_sync(0xffffffffu, mc.rec, q);
         const bool valid = cur * (uint32_t)C::TILE + 4u * (uint32_t)warp + (uint32_t)q < nnc32;
         uint32_t R = rec & 0x7Fu;
@@ -437,24 +520,24 @@ __global__ void __launch_bounds__(32 * NW + 32, SZX_EMINB) k_encode_f32(const fl
         cp_async_wait<0>();
         __syncwarp();  // the warp's own blocks are staged
         {   // R2 guard where classify could not prove it away: whole warp, one block at a time
-            const bool ng = valid && full && !(rec & 0x80u) && R < 32u;
+            const bool ng = valid && full && !(rec & 0x80u) && R < (uint32_t)TR::kFull;
             uint32_t gm = __ballot_sync(0xffffffffu, ng && ql == 0);
             while (gm) {
                 const int gl = __ffs(gm) - 1;
                 gm &= gm - 1;
-                float xw[4];
-                reinterpret_cast<uint4*>(xw)[0] = lds_u128(wib + (uint32_t)(gl >> 3) * 512u + 16u * swz16((uint32_t)lane));
-                const float gmu = __shfl_sync(0xffffffffu, mu, gl);
+                T xw[4];
+                warp_vals(wib, gl >> 3, xw);
+                const T gmu = TR::from(__shfl_sync(0xffffffffu, TR::bits(mu), gl));
                 const int gR = (int)__shfl_sync(0xffffffffu, R, gl);
-                const int fR = guard_R<float, 4>(xw, 4, gmu, gR, eb);
+                const int fR = guard_R<T, 4>(xw, 4, gmu, gR, eb);
                 if ((lane >> 3) == (gl >> 3)) R = (uint32_t)fR;
             }
         }
-        const bool fast = !__any_sync(0xffffffffu, valid && (!full || R >= 32u));
-        QEnc e;
+        const bool fast = !__any_sync(0xffffffffu, valid && (!full || R >= (uint32_t)TR::kFull));
+        typename std::conditional<sizeof(T) == 4, QEnc, QEnc64>::type e;
         uint32_t m8[16];
         uint32_t mexcl = 0;
-        uint32_t zex = 0;  // lane b < TILE: in-tile payload offset of block b
+        uint32_t zex = 0;   // lane b < TILE: in-tile payload offset of block b
         uint32_t rfin = 0;  // generic path: the final R of block kq in byte kq (after the R2 guard)
         auto generic = [&](bool pack) {
             // whole-warp encoder, one block at a time (raw blocks, the partial last block)
@@ -462,45 +545,47 @@ __global__ void __launch_bounds__(32 * NW + 32, SZX_EMINB) k_encode_f32(const fl
                 const int bj = warp * 4 + kq;
                 const bool bv = __shfl_sync(0xffffffffu, valid, 8 * kq);
                 const uint32_t bk = __shfl_sync(0xffffffffu, mk, 8 * kq);
-                const float bmu = __shfl_sync(0xffffffffu, mu, 8 * kq);
+                const T bmu = TR::from(__shfl_sync(0xffffffffu, TR::bits(mu), 8 * kq));
                 const uint32_t brec = __shfl_sync(0xffffffffu, rec, 8 * kq);
                 int bR = pack ? (int)((rfin >> (8 * kq)) & 0xFFu) : (int)__shfl_sync(0xffffffffu, R, 8 * kq);
                 if (!bv) {
                     if (!pack && lane == 0) s_z[bj] = 0u;
                     continue;
                 }
-                float xw[4];
-                uint32_t uu[4];
+                T xw[4];
+                typename TR::U uu[4];
                 LaneCode lc;
                 int cnt = 4, len = B;
                 if (bk < nBfull) {
-                    reinterpret_cast<uint4*>(xw)[0] = lds_u128(wib + (uint32_t)kq * 512u + 16u * swz16((uint32_t)lane));
+                    warp_vals(wib, kq, xw);
                 } else {
-                    cnt = load_lane<float, 4>(x, p.n, bk, lane, xw);
+                    cnt = load_lane<T, 4>(x, p.n, bk, lane, xw);
                     len = (int)(p.n - (uint64_t)bk * B);
                 }
-                if (!pack && bk >= nBfull && bR < 32) {
+                if (!pack && bk >= nBfull && bR < TR::kFull) {
                     // the partial last block: the R2 guard / escalation runs here (R2)
-                    encode_block<float, 4>(xw, cnt, len, bmu, bR, (brec & 0x80u) != 0, eb, uu, lc);
+                    encode_block<T, 4>(xw, cnt, len, bmu, bR, (brec & 0x80u) != 0, eb, uu, lc);
                     bR = lc.R;
                 } else {
-                    encode_known_R<float, 4>(xw, cnt, len, bR >= 32 ? 0.0f : bmu, bR, uu, lc);
+                    encode_known_R<T, 4>(xw, cnt, len, bR >= TR::kFull ? T(0) : bmu, bR, uu, lc);
                 }
                 if (!pack) {
                     rfin |= (uint32_t)bR << (8 * kq);
                     if (lane == 0) s_z[bj] = lc.z;
                 } else {
-                    pack_red<float, 4>(uu, lc, cnt, len, stg + __shfl_sync(0xffffffffu, zex, bj));
-                    if (lane == 0 && bR >= 32) mus[bk] = 0u;  // raw: mu = +0 (R15)
+                    pack_red<T, 4>(uu, lc, cnt, len, stg + __shfl_sync(0xffffffffu, zex, bj));
+                    if (lane == 0 && bR >= TR::kFull) mus[bk] = U(0);  // raw: mu = +0 (R15)
                 }
             }
         };
         if (fast) {
-            float xv[16];
+            T xv[16];
 #pragma unroll
-            for (int kq = 0; kq < 4; kq++)
-                reinterpret_cast<uint4*>(xv)[kq] = lds_u128(wib + (uint32_t)q * 512u + 16u * swz16(4u * ql + kq));
-            quarter_encode_f32(xv, mu, valid ? R : 9u, e, m8);
+            for (int kq = 0; kq < C::CPL; kq++)
+                reinterpret_cast<uint4*>(xv)[kq] =
+                    lds_u128(wib + (uint32_t)q * C::BW + 16u * swzc<C::CPL>((uint32_t)(C::CPL * ql + kq)));
+            if constexpr (sizeof(T) == 4) quarter_encode_f32(xv, mu, valid ? R : 9u, e, m8);
+            else quarter_encode_f64(xv, mu, valid ? R : 12u, e, m8);
             uint32_t incl = shfl_up_add8e<1>(e.msum);
             incl = shfl_up_add8e<2>(incl);
             incl = shfl_up_add8e<4>(incl);
@@ -517,20 +602,23 @@ __global__ void __launch_bounds__(32 * NW + 32, SZX_EMINB) k_encode_f32(const fl
             const uint32_t zl = lane < C::TILE ? s_z[lane] : 0u;
             const uint32_t incl = warp_incl_scan(zl);
             const uint32_t zoff = __shfl_sync(0xffffffffu, incl - zl, j);
-            const uint32_t T = __shfl_sync(0xffffffffu, incl, 31);
+            const uint32_t T_ = __shfl_sync(0xffffffffu, incl, 31);
             if (warp == 0) {
                 const uint32_t ncl = cur * (uint32_t)C::TILE + (uint32_t)lane;
                 if (lane < C::TILE && ncl < nnc32) zsize[ncl] = (uint16_t)zl;
-                if (lane == 0) st_relaxed(&p.status_e[cur], kFlagAgg | T);  // the tile's size, for the scanner
+                if (lane == 0) st_relaxed(&p.status_e[cur], kFlagAgg | T_);  // the tile's size, for the scanner
             }
             zex = incl - zl;
             if (fast) {
-                if (valid) quarter_pack_f32(e, m8, R, mexcl, stg + zoff);
+                if (valid) {
+                    if constexpr (sizeof(T) == 4) quarter_pack_f32(e, m8, R, mexcl, stg + zoff);
+                    else quarter_pack_f64(e, m8, R, mexcl, stg + zoff);
+                }
             } else {
                 generic(true);
             }
             if (tid == 0) {
-                s_T[slot] = T;
+                s_T[slot] = T_;
                 s_tile[slot] = cur;
             }
         }

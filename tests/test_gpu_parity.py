@@ -123,11 +123,13 @@ def test_parity_escalation_path():
         szx.set_r_bias(0)
 
 
-@pytest.mark.parametrize("rb,n", [(-3, 50_000), (-2, 50_000), (-3, 50_048), (-3, 128 * 16 * 5 + 77)])
-def test_parity_escalation_in_partial_last_block(rb, n):
+@pytest.mark.parametrize("rb,n,dt", [(-3, 50_000, np.float32), (-2, 50_000, np.float32), (-3, 50_048, np.float32),
+                                     (-3, 128 * 16 * 5 + 77, np.float32), (-3, 50_000, np.float64),
+                                     (-5, 128 * 16 * 3 + 5, np.float64)])
+def test_parity_escalation_in_partial_last_block(rb, n, dt):
     """The R2 guard / escalation must also run on the partial last block (a large offset makes
     the per-block proof fail, so every block is checked value by value; Formula 1)."""
-    x = synth.offset_field(n, 7, 3e3).numpy()
+    x = synth.offset_field(n, 7, 3e3, dtype=torch.float32 if dt == np.float32 else torch.float64).numpy()
     try:
         szx.set_r_bias(rb)
         got = szx.compress(torch.from_numpy(x).cuda(), 1e-4, "rel", 128).cpu().numpy()
