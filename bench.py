@@ -35,7 +35,7 @@ sys.path.insert(0, ROOT)
 METRIC = "SZx compress+decompress throughput, N*W / (T_compress + T_decompress)"
 UNIT = "GB/s"
 FIELD_NAMES = {0: "density", 1: "velocity", 2: "temperature"}
-NCU_NAME = {"k_decode": "k_decode_w", "k_encode": "k_encode_f32"}  # library timing label -> kernel name
+NCU_NAME = {"k_decode": "k_decode_w", "k_encode": "k_encode_fused"}  # library timing label -> kernel name
 FIELD_DESC = {0: "baryon-density-like exp(2.5g)", 1: "velocity-like 1e7 g", 2: "temperature-like 1e4 exp(0.7g)"}
 
 

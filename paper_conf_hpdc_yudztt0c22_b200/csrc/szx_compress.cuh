@@ -10,14 +10,17 @@
 //                        __ballot_sync, nonconstant-count scan (decoupled
 //                        look-back) that also writes the compacted list of
 //                        nonconstant block ids, and the stream header.
-//   k_encode       (K2+K3+K4 fused, persistent, warp-specialised) a producer
-//                        warp streams the nonconstant blocks of each tile
-//                        into a shared-memory ring with TMA bulk copies
-//                        (cp.async.bulk + mbarrier); 8 consumer warps encode
-//                        them: normalise, Formula 4 R, Formula 5 shift, lead
-//                        codes with __clz, R2 guard, warp scan of mid-byte
-//                        counts, tile look-back for the payload offset,
-//                        shared-memory packing, 16-byte stores.
+//   k_encode_fused (K2+K3+K4 fused, szx_encode.cuh; b = 128) persistent
+//                        cooperative kernel: compute warps take 4*NW-block
+//                        tiles by ticket, stage their own blocks with
+//                        cp.async, encode (normalise, Formula 4 R, Formula 5
+//                        shift, lead codes, R2 guard) and pack the tile in
+//                        shared memory; one scanner warp in CTA 0 turns the
+//                        published tile sizes into payload offsets (grid-wide
+//                        forward scan); the tile is copied out NS-1 tiles
+//                        later with 16-byte stores.
+//   k_enc_size / k_zscan / k_enc_write  the three-pass encoder for b != 128
+//                        (sizes, device-wide scan, write).
 //
 // Constant blocks are never read twice: after k_block_stats only the
 // nonconstant blocks are fetched again.  A warp owns one data block of
