@@ -182,12 +182,12 @@ CLayout clayout(uint64_t n, int W, uint32_t b) {
     CLayout L{};
     L.nB = cdiv(n, b);
     L.nW = cdiv(L.nB, 32);
-    L.nTB = cdiv(L.nB, kClassifyBlocks);
+    L.nTB = cdiv(L.nB, kClassifyMinBlocks);  // look-back words for the smallest classify tile
     L.nTC = cdiv(cdiv(L.nB, kWriteTile), 256);  // k_zscan CTAs (look-back status words)
     L.off_keys = 0;
     L.off_zero = 16;
     L.nTE = cdiv(L.nB, 4 * SZX_ENW) + 1;  // k_encode_f32 tiles (look-back status words)
-    L.zero_bytes = al16(16 + 8 * L.nTB + 8 * L.nTC + 16 * L.nTE);
+    L.zero_bytes = al16(16 + 16 * L.nTB + 8 * L.nTC + 16 * L.nTE);  // classify: 2 words per tile
     L.off_scal = L.off_zero + L.zero_bytes;
     L.off_stats = L.off_scal + 32;
     L.off_nclist = al16(L.off_stats + 2ull * W * L.nB);
@@ -211,7 +211,7 @@ Plan make_plan(const CLayout& L, uint8_t* ws, uint64_t n, szx_dtype_t dt, szx_eb
     p.range_keys = range_keys ? const_cast<uint64_t*>(range_keys) : reinterpret_cast<uint64_t*>(ws + L.off_keys);
     p.ctr = reinterpret_cast<uint32_t*>(ws + L.off_zero);
     p.status_b = reinterpret_cast<uint64_t*>(ws + L.off_zero + 16);
-    p.status_c = p.status_b + L.nTB;
+    p.status_c = p.status_b + 2 * L.nTB;
     p.status_e = p.status_c + L.nTC;
     p.prefix_e = p.status_e + L.nTE;
     p.eb_abs = reinterpret_cast<double*>(ws + L.off_scal);
@@ -317,9 +317,39 @@ void enqueue_stats(const void* d_in, const Plan& p, int want_range, cudaStream_t
 // nonconstant); CTAs beyond the device-side count exit at once.
 template <typename T, int VPL>
 void enqueue_encode(const void* d_in, const Plan& p, const CLayout& L, uint8_t* out, cudaStream_t s) {
-    kernel_occupancy(k_classify<T>, 0, 1);
     kernel_occupancy(k_zscan<Traits<T>::W>, 0, 1);
-    launch("k_classify", s, [&] { launch_pdl(k_classify<T>, dim3((unsigned)L.nTB), dim3(256), 0, s, p, out); });
+    {
+#ifndef SZX_CLS_COOP
+#define SZX_CLS_COOP 1   // classify: co-resident one-tile-per-CTA form when the tiles fit the grid
+#endif
+#ifndef SZX_CLS_TPSM
+#define SZX_CLS_TPSM 2   // classify (co-resident form): at most this many tiles per SM (0 = occupancy)
+#endif
+        // co-resident form: the smallest tile (blocks per thread) whose tile count
+        // fits the co-resident grid; else tiles by ticket with a look-back scan
+        bool done = false;
+        auto coop = [&](auto kern, int bpt) {
+            if (done) return;
+            const int occ = kernel_occupancy(kern, 0, 1);
+            uint64_t cap = (uint64_t)sm_count() * occ;
+            if (SZX_CLS_TPSM) cap = std::min<uint64_t>(cap, (uint64_t)SZX_CLS_TPSM * sm_count());
+            const uint64_t tiles = std::max<uint64_t>(1, cdiv(L.nB, 256ull * bpt));
+            if (tiles > cap) return;
+            done = true;
+            launch("k_classify", s, [&] { launch_coop(kern, dim3((unsigned)tiles), dim3(256), 0, s, p, out); });
+        };
+        if (SZX_CLS_COOP) {
+            coop(k_classify<T, 1, true>, 1);
+            coop(k_classify<T, 2, true>, 2);
+            coop(k_classify<T, 4, true>, 4);
+            coop(k_classify<T, 8, true>, 8);
+        }
+        if (!done) {
+            kernel_occupancy(k_classify<T, 8>, 0, 1);
+            const uint64_t grid = std::max<uint64_t>(1, cdiv(L.nB, (uint64_t)kClassifyBlocks));
+            launch("k_classify", s, [&] { launch_pdl(k_classify<T, 8>, dim3((unsigned)grid), dim3(256), 0, s, p, out); });
+        }
+    }
 #ifndef SZX_FUSED
 #define SZX_FUSED 1   // float32 b = 128: the fused single-pass encoder (szx_encode.cuh)
 #endif
@@ -349,6 +379,15 @@ void enqueue_encode(const void* d_in, const Plan& p, const CLayout& L, uint8_t* 
     });
     launch("k_zscan", s, [&] { launch_pdl(k_zscan<Traits<T>::W>, dim3((unsigned)L.nTC), dim3(256), 0, s, p, out); });
     using C = WriteCfg<T, VPL>;
+#ifndef SZX_DITEMS
+#define SZX_DITEMS 2        // decoder: target nonconstant work items per decode warp (tile split)
+#endif
+#ifndef SZX_DSPLIT
+#define SZX_DSPLIT 0        // decoder: force the tile split (1, 2, 4); 0 = by size
+#endif
+#ifndef SZX_ICTA_CHUNK
+#define SZX_ICTA_CHUNK 0    // decoder: index CTAs <= 256-tile chunks (measured slower: the index work per CTA grows)
+#endif
 #ifndef SZX_ICTA_PER_SM
 #define SZX_ICTA_PER_SM 1   // decoder CTAs per SM that run the index phase
 #endif
@@ -533,11 +572,18 @@ int enqueue_decompress(const void* d_in, uint64_t in_bytes, const szx_header_t* 
         // beside a concurrent kernel)
         auto go = [&](auto kern, const char* name) {
             const int occ = kernel_occupancy(kern, DecWCfg<T, V>::SMEM, 1);
-            uint64_t grid = cdiv(p.nWi, 8);
-            const uint64_t gcap = (uint64_t)sm_count() * occ;
+            const uint64_t gcap = std::min<uint64_t>((uint64_t)sm_count() * occ, kMaxDecodeGrid);
+            // small arrays: split each nonconstant tile into 2 or 4 work items so
+            // that every decode warp of the full grid gets a few (latency hiding)
+            const uint64_t want_items = (uint64_t)SZX_DITEMS * gcap * (DecWCfg<T, V>::NWARP - DecWCfg<T, V>::FILLW);
+            p.split = p.nWi >= want_items ? 1u : (p.nWi * 2 >= want_items ? 2u : 4u);
+            if (SZX_DSPLIT) p.split = SZX_DSPLIT;
+            uint64_t grid = cdiv(p.nWi * p.split, 8);
             if (grid > gcap) grid = gcap;
-            if (grid > kMaxDecodeGrid) grid = kMaxDecodeGrid;
-            p.n_icta = (uint32_t)std::min<uint64_t>(grid, (uint64_t)SZX_ICTA_PER_SM * sm_count());
+            // index CTAs: at most one per SM, and at most one 256-tile chunk each
+            // (fewer arrivals at the two grid-wide prefixes)
+            p.n_icta = (uint32_t)std::min<uint64_t>(std::min<uint64_t>(grid, (uint64_t)SZX_ICTA_PER_SM * sm_count()),
+                                                    SZX_ICTA_CHUNK ? cdiv(p.nWi, kIndexChunk) : grid);
             launch(name, s, [&] {
                 launch_coop(kern, dim3((unsigned)grid), dim3(256), DecWCfg<T, V>::SMEM, s, p, in,
                             reinterpret_cast<T*>(ybase));

@@ -262,22 +262,33 @@ __device__ inline void write_header(uint8_t* out, const Plan& p, double eb, uint
 }
 
 // ------------------------------------------------------------------ K1b
-// 256 threads x 8 blocks = 2048 blocks (64 bitmap words) per CTA tile.
-constexpr int kClassifyBlocks = 2048;
+// 256 threads x BPT blocks (8 BPT bitmap words) per CTA tile; BPT = 8 for
+// large fields, fewer for small ones so that the grid still covers the SMs
+// (the per-block work is a chain of dependent double-precision steps).
+constexpr int kClassifyBlocks = 2048;     // largest tile (BPT = 8)
+constexpr int kClassifyMinBlocks = 256;   // smallest tile (BPT = 1): sizes the look-back words
 
-template <typename T>
+// COOP = false: tiles by ticket, nonconstant-count scan by decoupled look-back
+// (large arrays).  COOP = true: one tile per CTA of a co-resident (cooperative)
+// grid and one grid-wide prefix instead: the look-back's depth grows with the
+// tile count, the prefix's does not (small arrays, where more, smaller tiles
+// shorten every thread's chain of dependent steps).
+template <typename T, int BPT, bool COOP = false>
 __global__ void __launch_bounds__(256) k_classify(Plan p, uint8_t* __restrict__ out) {
+    static_assert(BPT == 1 || BPT == 2 || BPT == 4 || BPT == 8, "BPT");
+    constexpr int CB = 256 * BPT;
     using TR = Traits<T>;
     using U = typename TR::U;
-    __shared__ uint64_t s_tile, s_base;
-    __shared__ uint32_t s_cnt[64], s_pre[64];
+    __shared__ uint64_t s_tile, s_base, s_agg;
+    __shared__ uint64_t s_w[32];
+    __shared__ uint32_t s_cnt[64], s_pre[64];  // [8 * BPT] used
     pdl_wait();
     pdl_trigger();
-    if (threadIdx.x == 0) s_tile = atomicAdd(&p.ctr[0], 1u);
+    if (!COOP && threadIdx.x == 0) s_tile = atomicAdd(&p.ctr[0], 1u);
     __syncthreads();
-    const uint64_t tile = s_tile;
+    const uint64_t tile = COOP ? (uint64_t)blockIdx.x : s_tile;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const uint64_t base = tile * kClassifyBlocks;
+    const uint64_t base = tile * CB;
     const double eb = eb_from_range(p.mode, p.eb_user, p.range_keys, p.eb_in);
     const int pe = expo_f64(eb);
     const U* stats = reinterpret_cast<const U*>(p.stats);
@@ -285,20 +296,20 @@ __global__ void __launch_bounds__(256) k_classify(Plan p, uint8_t* __restrict__ 
     U* mus = reinterpret_cast<U*>(out + p.off_mu);
 
     uint32_t ncmask = 0;
-    U rmu[8];
+    U rmu[BPT];
     uint32_t rrec[2] = {0u, 0u};  // per j: R_init | guard_proven << 7 (one byte each)
     // all eight blocks' keys first: the stores below (mu, bitmap) could alias the
     // stats for the compiler, which would otherwise serialise one load round trip
     // per block
-    U kmn[8], kmx[8];
+    U kmn[BPT], kmx[BPT];
 #pragma unroll
-    for (int j = 0; j < 8; j++) {
+    for (int j = 0; j < BPT; j++) {
         const uint64_t k = base + j * 256 + threadIdx.x;
         kmn[j] = k < p.nB ? stats[2 * k] : U(0);
         kmx[j] = k < p.nB ? stats[2 * k + 1] : U(0);
     }
 #pragma unroll
-    for (int j = 0; j < 8; j++) {
+    for (int j = 0; j < BPT; j++) {
         const uint64_t k = base + j * 256 + threadIdx.x;
         bool nc = false;
         rmu[j] = 0;
@@ -327,16 +338,28 @@ __global__ void __launch_bounds__(256) k_classify(Plan p, uint8_t* __restrict__ 
     }
     __syncthreads();
     if (warp == 0) {
-        const uint32_t c0 = s_cnt[2 * lane], c1 = s_cnt[2 * lane + 1];
+        const uint32_t c0 = 2 * lane < 8 * BPT ? s_cnt[2 * lane] : 0u;
+        const uint32_t c1 = 2 * lane + 1 < 8 * BPT ? s_cnt[2 * lane + 1] : 0u;
         const uint32_t incl = warp_incl_scan(c0 + c1);
         const uint32_t ex = incl - c0 - c1;
         s_pre[2 * lane] = ex;
         s_pre[2 * lane + 1] = ex + c0;
         const uint32_t agg = __shfl_sync(0xffffffffu, incl, 31);
-        const uint64_t G = lookback_exclusive(p.status_b, tile, agg);
-        if (lane == 0) {
-            s_base = G;
-            const uint64_t ntiles = (p.nB + kClassifyBlocks - 1) / kClassifyBlocks;
+        if (lane == 0) s_agg = agg;
+        if (!COOP) {
+            const uint64_t G = lookback_exclusive(p.status_b, tile, agg);
+            if (lane == 0) s_base = G;
+        }
+    }
+    if (COOP) {
+        __syncthreads();
+        const uint64_t G = grid_excl_prefix(p.status_b, p.status_b + gridDim.x, &p.ctr[1], s_agg, s_w, gridDim.x);
+        if (threadIdx.x == 0) s_base = G;
+    }
+    if (threadIdx.x == 0) {
+        {
+            const uint64_t G = s_base, agg = s_agg;
+            const uint64_t ntiles = (p.nB + CB - 1) / CB;
             if (tile == ntiles - 1) {
                 const uint64_t nnc = G + agg;
                 *p.nnc = nnc;
@@ -359,7 +382,7 @@ __global__ void __launch_bounds__(256) k_classify(Plan p, uint8_t* __restrict__ 
     const uint64_t G = s_base;
     U* ncmu = reinterpret_cast<U*>(p.ncmu);
 #pragma unroll
-    for (int j = 0; j < 8; j++) {
+    for (int j = 0; j < BPT; j++) {
         const bool nc = (ncmask >> j) & 1u;
         const uint32_t word = __ballot_sync(0xffffffffu, nc);
         if (nc) {

@@ -46,6 +46,7 @@ struct DPlan {
     uint64_t* tbase;           // [nW + 1]  payload offset of each tile (tbase[nW] = total)
     int32_t* err;              // 0 ok, else SZX_ECORRUPT
     uint32_t n_icta;           // CTAs that run the index phase (<= gridDim.x)
+    uint32_t split;            // work items per nonconstant tile (1, 2 or 4: 32/split blocks each)
     // quality variant only: the original values, indexed
     // like y, and the accumulators {max |x-x'| (double bits), sum (x-x')^2
     // (double), dkey(min finite x), ~dkey(max finite x)}, initialised by the host
@@ -988,9 +989,13 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 8 && VPL == 4) ? 2 : SZX_DM
     // grid barrier: tiles are decoded by whichever warp grabs them
     // (one CTA per SM at most: fewer arrivals at the two grid-wide prefixes)
     if (blockIdx.x < p.n_icta) index_phase<W>(p, in, hd, reinterpret_cast<uint16_t*>(dsm), s_w);
+    // (The fill warps need only the bitmap and mu, but starting them before
+    // the barrier measured slower: their traffic stretches the latency-bound
+    // index phase -- NYX velocity index 16 -> 22 us, Hurricane decode +8 us.)
     grid_barrier(&p.ctr[2]);
     SZX_TL(1);
     const int lane = threadIdx.x & 31;
+    const int wid = threadIdx.x >> 5;
     const uint32_t* bm = reinterpret_cast<const uint32_t*>(in + kHeaderBytes);
     const uint16_t* zs = reinterpret_cast<const uint16_t*>(in + hd.off_zs);
     const U* mus = reinterpret_cast<const U*>(in + p.off_mu);
@@ -1047,8 +1052,6 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 8 && VPL == 4) ? 2 : SZX_DM
             mul = mn;
         }
     };
-    const uint32_t n_nct = *p.n_nctile;
-
     auto load_meta = [&](uint64_t t, TileMeta<U>& m) {
         uint32_t word = bm[t];
         if (t == p.nW - 1 && (p.nB & 31)) word &= (1u << (p.nB & 31)) - 1u;
@@ -1087,14 +1090,14 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 8 && VPL == 4) ? 2 : SZX_DM
         r.ok = ok && __all_sync(0xffffffffu, zok) && __shfl_sync(0xffffffffu, r.zincl, 31) == m.end - m.base;
         return r;
     };
-    // the segment starting at rank r0: as many blocks as fit SLOT - 16 bytes
-    auto seg_from = [&](const TileZ& z, uint32_t r0) -> SegT {
+    // the segment starting at rank r0: as many blocks of ranks < rmax as fit SLOT - 16 bytes
+    auto seg_from = [&](const TileZ& z, uint32_t r0, uint32_t rmax) -> SegT {
         SegT sg;
         sg.r0 = r0;
         sg.off0 = r0 ? __shfl_sync(0xffffffffu, z.zincl, r0 - 1) : 0u;
-        const bool fits = (uint32_t)lane >= r0 && (uint32_t)lane < z.cnt && z.zincl - sg.off0 <= (uint32_t)(C::SLOT - 16);
+        const bool fits = (uint32_t)lane >= r0 && (uint32_t)lane < rmax && z.zincl - sg.off0 <= (uint32_t)(C::SLOT - 16);
         sg.r1 = r0 + __popc(__ballot_sync(0xffffffffu, fits));
-        if (sg.r1 == r0 && r0 < z.cnt) sg.r1 = r0 + 1;  // (corrupt sizes: validated separately)
+        if (sg.r1 == r0 && r0 < rmax) sg.r1 = r0 + 1;  // (corrupt sizes: validated separately)
         return sg;
     };
     // cp.async the segment's bytes into slot `sl`
@@ -1112,15 +1115,28 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 8 && VPL == 4) ? 2 : SZX_DM
         }
     };
     // dynamic assignment over the list of tiles holding nonconstant blocks
-    // (their cost varies far more than the fill's)
-    auto grab = [&]() -> uint64_t {
-        uint32_t v = 0xFFFFFFFFu;
+    // (their cost varies far more than the fill's); a work item is one of the
+    // `split` equal parts of such a tile (small arrays: more warps in flight)
+    const uint32_t split = p.split;
+    uint32_t n_items = 0;  // set once the index is complete
+    auto grab = [&](uint32_t& part) -> uint64_t {
+        uint32_t v = 0xFFFFFFFFu, pt = 0;
         if (lane == 0) {
             const uint32_t i = atomicAdd(&p.ctr[4], 1u);
-            if (i < n_nct) v = p.nctile[i];
+            if (i < n_items) {
+                v = p.nctile[i / split];
+                pt = i % split;
+            }
         }
         v = __shfl_sync(0xffffffffu, v, 0);
+        part = __shfl_sync(0xffffffffu, pt, 0);
         return v == 0xFFFFFFFFu ? p.nW : (uint64_t)v;
+    };
+    // ranks [ra, rb) of the tile's nonconstant blocks that lie in part `part`
+    auto part_ranks = [&](uint32_t word, uint32_t part, uint32_t& ra, uint32_t& rb) {
+        const uint32_t lo = part * (32u / split), hi = lo + 32u / split;
+        ra = __popc(word & ((1u << lo) - 1u));
+        rb = hi >= 32u ? __popc(word) : __popc(word & ((1u << hi) - 1u));
     };
     // decode the blocks of ranks [r0, r1) of a full tile from the staged slot
     auto decode_seg = [&](uint64_t t, const TileMeta<U>& m, const TileZ& z, const SegT& sg, int sl) {
@@ -1337,41 +1353,46 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 8 && VPL == 4) ? 2 : SZX_DM
     };
 
     auto nc_loop = [&]() {
-        uint64_t t = grab();
+        n_items = *p.n_nctile * split;
+        uint32_t part, pn;
+        uint64_t t = grab(part);
         if (t >= p.nW) return;
         TileMeta<U> cur, nx;
         load_meta(t, cur);
         load_zl(cur);
         TileZ cz = tile_z(cur);
-        SegT sg = seg_from(cz, 0);
+        uint32_t ra, rb, na = 0, nb = 0;
+        part_ranks(cur.word, part, ra, rb);
+        SegT sg = seg_from(cz, ra, rb);
         const bool cfull0 = t < nW_full;
-        if (cfull0 && cz.ok && cz.cnt) stage_seg(cur, cz, sg, 0);
+        if (cfull0 && cz.ok && rb > ra) stage_seg(cur, cz, sg, 0);
         cp_async_commit();
-        uint64_t tn = grab();
+        uint64_t tn = grab(pn);
         if (tn < p.nW) load_meta(tn, nx);
         int sl = 0;
         while (t < p.nW) {
             const bool cfull = t < nW_full;
-            if (!cz.ok && lane == 0) set_corrupt(p.err);
-            // the next work item: the rest of this tile, or the next tile
-            bool next_same = cfull && cz.ok && sg.r1 < cz.cnt;
+            if (!cz.ok && lane == 0 && part == 0) set_corrupt(p.err);
+            // the next work item: the rest of this part, or the next part / tile
+            bool next_same = cfull && cz.ok && sg.r1 < rb;
             TileZ nz = cz;
             SegT ns = sg;
             if (next_same) {
-                ns = seg_from(cz, sg.r1);
+                ns = seg_from(cz, sg.r1, rb);
                 stage_seg(cur, cz, ns, sl ^ 1);
             } else if (tn < p.nW) {
                 load_zl(nx);
                 nz = tile_z(nx);
-                ns = seg_from(nz, 0);
-                if (tn < nW_full && nz.ok && nz.cnt) stage_seg(nx, nz, ns, sl ^ 1);
+                part_ranks(nx.word, pn, na, nb);
+                ns = seg_from(nz, na, nb);
+                if (tn < nW_full && nz.ok && nb > na) stage_seg(nx, nz, ns, sl ^ 1);
             }
             cp_async_commit();
             cp_async_wait<1>();
             __syncwarp();
             if (cz.ok) {
                 if (cfull) decode_seg(t, cur, cz, sg, sl);
-                else decode_partial(t, cur, cz);
+                else if (part == 0) decode_partial(t, cur, cz);  // the partial tile: whole, by part 0
             }
             __syncwarp();  // slot `sl` is refilled by the item after next
             sl ^= 1;
@@ -1379,11 +1400,14 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 8 && VPL == 4) ? 2 : SZX_DM
                 sg = ns;
             } else {
                 t = tn;
+                part = pn;
+                ra = na;
+                rb = nb;
                 cur = nx;
                 cz = nz;
                 sg = ns;
                 if (t < p.nW) {
-                    tn = grab();
+                    tn = grab(pn);
                     if (tn < p.nW) load_meta(tn, nx);
                 }
             }
@@ -1394,7 +1418,7 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 8 && VPL == 4) ? 2 : SZX_DM
     // the split adapts to the field's fraction of nonconstant blocks.  (Decode
     // warps joining the fill as well, SZX_SWITCH = 3, measured slower: more
     // concurrent fill streams cut the write rate -- NYX density 107 -> 149 us.)
-    if ((int)(threadIdx.x >> 5) < C::FILLW) {
+    if (wid < C::FILLW) {
         fill_loop();
         SZX_TL(2);
         if (SZX_SWITCH & 2) nc_loop();

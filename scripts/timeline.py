@@ -22,7 +22,13 @@ import synth
 
 field = int(os.environ.get("FIELD", "0"))
 fillw = int(os.environ.get("FILLW", "2"))
-x = synth.nyx_like(field, n=512, device="cuda").reshape(-1).contiguous()
+cfg = os.environ.get("CFG", "nyx")  # nyx | cesm | hurricane
+if cfg == "cesm":
+    x = synth.cesm_like(0, device="cuda").reshape(-1).contiguous()
+elif cfg == "hurricane":
+    x = synth.hurricane_like(0, device="cuda").reshape(-1).contiguous()
+else:
+    x = synth.nyx_like(field, n=512, device="cuda").reshape(-1).contiguous()
 c = szx.Codec(x.numel(), torch.float32, 128)
 y = torch.empty_like(x)
 c.compress_async(x, 1e-3, "rel")
@@ -54,7 +60,7 @@ def q(a):
 
 
 print(json.dumps({
-    "field": field, "ctas": ctas,
+    "cfg": cfg, "field": field, "ctas": ctas,
     "entry": q(us[:, :, 0]),
     # warp 0 only: its stamp follows the barrier's polling loop; the other
     # warps' stamp may be scheduled before the barrier's second bar.sync
