@@ -1334,4 +1334,11 @@ int szx_debug_timeline(uint64_t* h_dst, uint64_t n) {
     return cudaMemcpyFromSymbol(h_dst, szx::g_tl, 8 * (n < cap ? n : cap)) == cudaSuccess ? SZX_OK : SZX_ECUDA;
 }
 #endif
+#if SZX_ETIMELINE
+// diagnostic timing builds only: the fused encoder's per-tile timeline (4 x u64 per tile)
+int szx_debug_enc_timeline(uint64_t* h_dst, uint64_t n) {
+    const uint64_t cap = sizeof(szx::g_etl) / sizeof(uint64_t);
+    return cudaMemcpyFromSymbol(h_dst, szx::g_etl, 8 * (n < cap ? n : cap)) == cudaSuccess ? SZX_OK : SZX_ECUDA;
+}
+#endif
 }  // extern "C"

@@ -46,6 +46,25 @@ namespace szx {
 #define SZX_ENS 3     // staging slots per encoder CTA (tiles in flight)
 #endif
 
+// Diagnostic timing builds only (-DSZX_ETIMELINE=1, scripts/enc_timeline.py):
+// %globaltimer per tile at publish, prefix written, retire start / end.
+#ifndef SZX_ETIMELINE
+#define SZX_ETIMELINE 0
+#endif
+#if SZX_ETIMELINE
+constexpr int kEtlTiles = 1 << 17;
+__device__ uint64_t g_etl[kEtlTiles * 4];
+__device__ inline uint64_t gtimer() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t)::"memory");
+    return t;
+}
+#define SZX_ETL(tile, k) \
+    do { if ((tile) < (uint64_t)kEtlTiles) g_etl[(uint64_t)(tile) * 4 + (k)] = gtimer(); } while (0)
+#else
+#define SZX_ETL(tile, k) do { } while (0)
+#endif
+
 // 16-byte chunk c (0..31) of a staged block sits at swz16(c): lane ql of a
 // quarter reads chunks 4 ql .. 4 ql + 3, and the 8 lanes of one LDS.128 phase
 // then hit 8 distinct 16-byte bank groups
@@ -174,7 +193,10 @@ __device__ inline void tile_scanner(const uint64_t* status, uint64_t* prefix, ui
         const uint64_t lex = run + incl - loc;
 #pragma unroll
         for (int k = 0; k < K; k++)
-            if (K * lane + k < nready) st_relaxed(&prefix[base + K * lane + k], (1ull << 63) | (lex + pre[k]));
+            if (K * lane + k < nready) {
+                st_relaxed(&prefix[base + K * lane + k], (1ull << 63) | (lex + pre[k]));
+                SZX_ETL(base + K * lane + k, 1);
+            }
         run += __shfl_sync(0xffffffffu, incl, 31);
         base += (uint64_t)nready;
         if (nready == WIN) {
@@ -448,6 +470,7 @@ __global__ void __launch_bounds__(32 * NW + 32, sizeof(T) == 4 ? SZX_EMINB : 3) 
     auto retire = [&](uint32_t kk) {
         const int sl = (int)(kk % NS);
         if (tid == 0) {
+            SZX_ETL(s_tile[sl], 2);
             uint64_t v;
             uint32_t ns = 32;
             while (!((v = ld_relaxed(&p.prefix_e[s_tile[sl]])) >> 63)) {
@@ -458,6 +481,7 @@ __global__ void __launch_bounds__(32 * NW + 32, sizeof(T) == 4 ? SZX_EMINB : 3) 
         }
         bar_compute(C::NTC);
         copy_out_tile<C::NTC>(slot_addr(sl), out + off_pl + s_excl[sl], s_T[sl]);
+        if (tid == 0) SZX_ETL(s_tile[sl], 3);
         // (the slot is zeroed when it is reused, NS - 1 tiles later)
     };
     // metadata of this warp's 4 blocks of tile t (lanes 0-3); the values are staged by
@@ -606,7 +630,10 @@ __global__ void __launch_bounds__(32 * NW + 32, sizeof(T) == 4 ? SZX_EMINB : 3) 
             if (warp == 0) {
                 const uint32_t ncl = cur * (uint32_t)C::TILE + (uint32_t)lane;
                 if (lane < C::TILE && ncl < nnc32) zsize[ncl] = (uint16_t)zl;
-                if (lane == 0) st_relaxed(&p.status_e[cur], kFlagAgg | T_);  // the tile's size, for the scanner
+                if (lane == 0) {
+                    st_relaxed(&p.status_e[cur], kFlagAgg | T_);  // the tile's size, for the scanner
+                    SZX_ETL(cur, 0);
+                }
             }
             zex = incl - zl;
             if (fast) {
