@@ -382,6 +382,9 @@ void enqueue_encode(const void* d_in, const Plan& p, const CLayout& L, uint8_t* 
 #ifndef SZX_DITEMS
 #define SZX_DITEMS 2        // decoder: target nonconstant work items per decode warp (tile split)
 #endif
+#ifndef SZX_DTS
+#define SZX_DTS 1           // decoder: thread-serial tiles on dense float32 b = 128 streams
+#endif
 #ifndef SZX_DSPLIT
 #define SZX_DSPLIT 0        // decoder: force the tile split (1, 2, 4); 0 = by size
 #endif
@@ -578,6 +581,10 @@ int enqueue_decompress(const void* d_in, uint64_t in_bytes, const szx_header_t* 
             const uint64_t want_items = (uint64_t)SZX_DITEMS * gcap * (DecWCfg<T, V>::NWARP - DecWCfg<T, V>::FILLW);
             p.split = p.nWi >= want_items ? 1u : (p.nWi * 2 >= want_items ? 2u : 4u);
             if (SZX_DSPLIT) p.split = SZX_DSPLIT;
+            // dense float32 b = 128 streams: the thread-serial tile decoder (a
+            // performance choice only; the device validates the stream itself)
+            p.ts = (SZX_DTS && sizeof(T) == 4 && V == 4 && !d_ref && p.split == 1 && kb0 == 0 &&
+                    kb1 == L.nB && 4 * h->n_nonconst >= 3 * L.nB) ? 1u : 0u;
             uint64_t grid = cdiv(p.nWi * p.split, 8);
             if (grid > gcap) grid = gcap;
             // index CTAs: at most one per SM, and at most one 256-tile chunk each

@@ -47,6 +47,7 @@ struct DPlan {
     int32_t* err;              // 0 ok, else SZX_ECORRUPT
     uint32_t n_icta;           // CTAs that run the index phase (<= gridDim.x)
     uint32_t split;            // work items per nonconstant tile (1, 2 or 4: 32/split blocks each)
+    uint32_t ts;               // dense float32 b = 128 stream: lane-per-block (thread-serial) tile decoder
     // quality variant only: the original values, indexed
     // like y, and the accumulators {max |x-x'| (double bits), sum (x-x')^2
     // (double), dkey(min finite x), ~dkey(max finite x)}, initialised by the host
@@ -922,7 +923,22 @@ struct DecWCfg {
 #define SZX_SWITCH 2
 #endif
     static constexpr int FILLW = SZX_FILLW;         // fill warps per CTA (the rest decode)
-    static constexpr int SMEM = NWARP * 2 * SLOT_ALLOC;
+#ifndef SZX_TSUNC
+#define SZX_TSUNC 0  // thread-serial window: unpredicated look-ahead load (measured slower)
+#endif
+#ifndef SZX_TSPF
+#define SZX_TSPF 0   // thread-serial tiles: bulk L2 prefetch of the next tile's payload
+#endif
+#ifndef SZX_DREGION
+#define SZX_DREGION 9216
+#endif
+    // per-warp shared region: the two staging slots of the segment decoder, or
+    // (thread-serial tiles) a 1 KB transpose buffer + one staging area + over-read pad
+    static constexpr int REGION = SZX_DREGION > 2 * SLOT_ALLOC ? SZX_DREGION : 2 * SLOT_ALLOC;
+    static constexpr int TS_TB = 1024;               // transpose buffer: 32 blocks x 8 values
+    static constexpr int TS_PAD = 576;               // > 12 + 128 x 4 bytes a corrupt lane may over-read
+    static constexpr int TS_STAGE = REGION - TS_TB - TS_PAD;
+    static constexpr int SMEM = NWARP * REGION;
     static_assert(SMEM >= kIndexChunk * 32 * 2, "index-phase scratch aliases the slots");
 };
 
@@ -948,6 +964,91 @@ __device__ uint64_t g_tl[kTlCtas * 8 * 4];
     do {          \
     } while (0)
 #endif
+
+
+// ---- thread-serial tile decoder (float32, b = 128): lane j decodes block j
+// of a 32-block tile alone, Fig. 10's five steps value after value
+// -- no cross-lane scans: the lead-byte chain is the lane's own
+// `prev`, the mid-bytes come from a 3-word window sliding over the block's
+// staged payload.  Every 8 values the warp transposes its 32 x 8 values
+// through shared memory and stores them as 32-byte block segments.
+// a: shared address of the lane's payload [R][32 code bytes][mid-bytes];
+// tb: 1 KB transpose buffer; yt: the tile's first output value; word: the
+// tile's nonconstant bitmap (lanes of constant blocks run on dummy input and
+// store nothing).  Returns false (this lane) on a size mismatch.
+template <bool RAWOK>
+__device__ __forceinline__ bool ts_decode_f32(uint32_t a, uint32_t R, uint32_t zz, float mu, uint32_t tb,
+                                              float* __restrict__ yt, uint32_t word) {
+    const int lane = threadIdx.x & 31;
+    const bool raw = RAWOK && R >= 32u;
+    const uint32_t s = raw ? 0u : ((8u - (R & 7u)) & 7u);
+    const uint32_t r8 = raw ? 32u : R + s;              // kept bits, whole bytes: 16, 24 or 32
+    const uint32_t pdrop = launder(1u << (32u - r8));   // (shifts as IMADs on the FMA pipe)
+    const uint32_t ps = launder(1u << s);
+    const uint32_t fix = r8 == 16u ? 0x55555555u : 0u;  // req = 2: code 3 copies 2 bytes
+    const uint32_t mb = a + 33u, wp = mb & ~3u, pos0 = 8u * (mb & 3u);
+    // window (lo, hi, nx) = words k, k+1, k+2 of the run from wp; pos = absolute
+    // bit position from wp (lo holds bits [32 k, 32 k + 32)), lim = 32 (k + 1)
+    uint32_t lo = lds_u32(wp), hi = lds_u32(wp + 4), nx = lds_u32(wp + 8);
+    uint32_t pos = pos0, lim = 32u, prev = 0;
+    const uint32_t wp8 = wp + 8u;
+    const uint32_t sw = ((uint32_t)lane >> 2) & 1u;     // transpose swizzle (bank-conflict free)
+#pragma unroll 1
+    for (int g = 0; g < 8; g++) {
+        const uint32_t cb = a + 1u + 4u * (uint32_t)g;  // this group's 16 lead codes (4 bytes)
+        uint32_t cw = __funnelshift_r(lds_u32(cb & ~3u), lds_u32((cb & ~3u) + 4), 8u * cb);
+        cw ^= cw & (cw >> 1) & fix;
+#pragma unroll
+        for (int h = 0; h < 2; h++) {
+            float o[8];
+#pragma unroll
+            for (int i = 0; i < 8; i++) {
+                const int ii = 8 * h + i;
+                // step 2: c8 = 8 x bytes copied from the previous value; step 3: m8 = 8 x mid-bytes
+                const uint32_t c8 = ii == 0 ? (cw << 3) & 24u : ii == 1 ? (cw << 1) & 24u : (cw >> (2 * ii - 3)) & 24u;
+                const uint32_t nm = 0xFFFFFFFFu >> c8;
+                const uint32_t m8 = r8 - c8;
+                const uint32_t mid = __funnelshift_r(lo, hi, pos);
+                const uint32_t w = bitsel(prev, mid * pdrop, nm);  // steps 2-4
+                prev = w;
+                o[i] = raw ? __uint_as_float(w) : __fadd_rn(__uint_as_float(w * ps), mu);  // step 5
+                pos += m8;
+#if SZX_TSUNC
+                // slide one word (m8 <= 32: at most one per value); nx is re-read
+                // every value (unpredicated: no move of a just-loaded register)
+                const bool sl = pos >= lim;
+                lim += sl ? 32u : 0u;
+                lo = sl ? hi : lo;
+                hi = sl ? nx : hi;
+                nx = lds_u32(wp8 + (lim >> 3) - 4u);
+#else
+                if (pos >= lim) {  // slide one word (m8 <= 32: at most one per value)
+                    lim += 32u;
+                    lo = hi;
+                    hi = nx;
+                    nx = lds_u32(wp8 + (lim >> 3) - 4u);  // word k + 2 of the new window
+                }
+#endif
+            }
+            const uint32_t row = tb + 32u * (uint32_t)lane;
+            asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(row + 16u * sw), "r"(__float_as_uint(o[0])),
+                         "r"(__float_as_uint(o[1])), "r"(__float_as_uint(o[2])), "r"(__float_as_uint(o[3])) : "memory");
+            asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(row + 16u * (sw ^ 1u)), "r"(__float_as_uint(o[4])),
+                         "r"(__float_as_uint(o[5])), "r"(__float_as_uint(o[6])), "r"(__float_as_uint(o[7])) : "memory");
+            __syncwarp();
+#pragma unroll
+            for (int k = 0; k < 2; k++) {
+                const uint32_t b = ((uint32_t)lane >> 1) + 16u * (uint32_t)k, c = (uint32_t)lane & 1u;
+                const uint4 v = lds_u128(tb + 32u * b + 16u * (c ^ ((b >> 2) & 1u)));
+                if ((word >> b) & 1u)
+                    st_out16(reinterpret_cast<uint4*>(yt + 128u * b + 16u * (uint32_t)g + 8u * (uint32_t)h + 4u * c), v);
+            }
+            __syncwarp();
+        }
+    }
+    // the block's mid-bytes end exactly at its zsize
+    return pos - pos0 == 8u * (zz - 33u);
+}
 
 // Per-tile metadata a warp needs before it can store anything.
 template <typename U>
@@ -1002,7 +1103,7 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 8 && VPL == 4) ? 2 : SZX_DM
     const uint8_t* pl = in + hd.off_pl;
     const uintptr_t lim = reinterpret_cast<uintptr_t>(in) + p.in_bytes;
     const uint64_t nW_full = p.n / ((uint64_t)TB * B);
-    const uint32_t slot0 = smem_u32(dsm + (threadIdx.x >> 5) * 2 * C::SLOT_ALLOC);
+    const uint32_t slot0 = smem_u32(dsm + (threadIdx.x >> 5) * C::REGION);
     // blocks of tile t inside the requested range [kb0, kb1)
     auto rmask = [&](uint64_t t) -> uint32_t {
         uint32_t m = 0xFFFFFFFFu;
@@ -1050,6 +1151,36 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 8 && VPL == 4) ? 2 : SZX_DM
             t = tn;
             word = wn;
             mul = mn;
+        }
+    };
+
+    // Dense streams (p.ts): every warp decodes first, then fills the few
+    // constant blocks; tiles are claimed 32 at a time and skipped with one
+    // ballot when they hold no constant block.
+    auto fill_ts = [&]() {
+        for (;;) {
+            uint32_t c = 0;
+            if (lane == 0) c = atomicAdd(&p.ctr[1], 1u);
+            const uint64_t t0 = p.t_lo + 32ull * __shfl_sync(0xffffffffu, c, 0);
+            if (t0 >= fill_end) break;
+            const uint64_t tl = t0 + lane;
+            const uint32_t cm = tl < fill_end ? ~bm[tl] & rmask(tl) : 0u;  // constant blocks of tile tl
+            for (uint32_t todo = __ballot_sync(0xffffffffu, cm != 0u); todo; todo &= todo - 1) {
+                const int jt = __ffs(todo) - 1;
+                const uint64_t t = t0 + jt;
+                const uint32_t m = __shfl_sync(0xffffffffu, cm, jt);
+                const U mul = mus[t * TB + lane];
+                V* yq = reinterpret_cast<V*>(y + t * TB * B + lane * VPL);
+                for (uint32_t mm = m; mm; mm &= mm - 1) {
+                    const int j = __ffs(mm) - 1;
+                    const U mb = __shfl_sync(0xffffffffu, mul, j);
+                    T v[VPL];
+#pragma unroll
+                    for (int q = 0; q < VPL; q++) v[q] = TR::from(mb);
+#pragma unroll
+                    for (int q = 0; q < NV; q++) st_out(yq + j * QB + q, reinterpret_cast<const V*>(v)[q]);
+                }
+            }
         }
     };
     auto load_meta = [&](uint64_t t, TileMeta<U>& m) {
@@ -1352,6 +1483,89 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 8 && VPL == 4) ? 2 : SZX_DM
         }
     };
 
+
+    // Dense float32 b = 128 streams (p.ts): tiles with >= 24 nonconstant blocks
+    // whose payload fits the staging area go to the thread-serial decoder, the
+    // others to the segment decoder (not pipelined here); the whole tile is
+    // staged, then decoded -- the warps of the SM hide each other's staging.
+    auto ts_loop = [&]() {
+        if constexpr (sizeof(T) == 4 && VPL == 4 && !QUAL) {
+            // software pipeline over tiles: at tile k the ticket of tile k+2 is
+            // in flight (atomic, then its list entry), the metadata of tile k+1
+            // is loaded and its zsizes are being read -- none of these global
+            // latencies is waited for inside the tile that issues them
+            n_items = *p.n_nctile;
+            auto tile_of = [&](uint32_t i) -> uint64_t { return i < n_items ? (uint64_t)p.nctile[i] : p.nW; };
+            uint32_t i0 = 0, i1 = 0;
+            if (lane == 0) { i0 = atomicAdd(&p.ctr[4], 1u); i1 = atomicAdd(&p.ctr[4], 1u); }
+            uint64_t t = tile_of(__shfl_sync(0xffffffffu, i0, 0));
+            uint64_t tn = tile_of(__shfl_sync(0xffffffffu, i1, 0));
+            TileMeta<U> cur, nx;
+            if (t < p.nW) {
+                load_meta(t, cur);
+                load_zl(cur);
+            }
+            if (tn < p.nW) load_meta(tn, nx);
+            const uint32_t region = slot0, tb = region, sa = region + C::TS_TB;
+            while (t < p.nW) {
+                uint32_t iraw = 0;  // the ticket of the tile after next (read at the end of this tile)
+                if (lane == 0) iraw = atomicAdd(&p.ctr[4], 1u);
+                const TileZ cz = tile_z(cur);
+                if (tn < p.nW) load_zl(nx);
+                const uint64_t bytes = cur.end - cur.base;
+                if (!cz.ok) {
+                    if (lane == 0) set_corrupt(p.err);
+                } else if (t < nW_full && cz.cnt >= 24u && bytes + 15u <= (uint64_t)C::TS_STAGE) {
+                    // stage the tile's payload (16-byte chunks), then decode a block per lane
+                    const uintptr_t g0 = reinterpret_cast<uintptr_t>(pl + cur.base);
+                    const uintptr_t gA = g0 & ~uintptr_t(15);
+                    const uintptr_t gE = (reinterpret_cast<uintptr_t>(pl + cur.end) + 15) & ~uintptr_t(15);
+                    for (uintptr_t ga = gA + 16 * lane; ga < gE; ga += 16 * 32) {
+                        const uintptr_t rem = lim - ga;
+                        cp_async16_zfill(sa + (uint32_t)(ga - gA), reinterpret_cast<const void*>(ga), rem < 16 ? (uint32_t)rem : 16u);
+                    }
+                    cp_async_commit();
+                    const uint32_t sbase = sa + (uint32_t)(g0 & 15);
+                    const bool has = (cur.word >> lane) & 1u;
+                    const uint32_t rank = __popc(cur.word & ((1u << lane) - 1u));
+                    const uint32_t offl = __shfl_sync(0xffffffffu, cz.zincl - cz.zl, rank & 31u);
+                    const uint32_t zz = __shfl_sync(0xffffffffu, cz.zl, rank & 31u);
+                    const uint32_t a = has ? sbase + offl : sbase;
+                    cp_async_wait<0>();
+                    __syncwarp();
+                    const uint32_t R = has ? lds_u8(a) : 9u;
+                    const bool bad = R < 9u || R > 32u;
+                    float* yt = reinterpret_cast<float*>(y) + t * TB * B;
+                    const float mu = __uint_as_float((uint32_t)cur.mul);
+                    bool ok;
+                    if (__any_sync(0xffffffffu, R >= 32u)) ok = ts_decode_f32<true>(a, R, has ? zz : 33u, mu, tb, yt, cur.word);
+                    else ok = ts_decode_f32<false>(a, R, has ? zz : 33u, mu, tb, yt, cur.word);
+                    if (has && (bad || !ok)) set_corrupt(p.err);
+                } else if (t < nW_full) {
+                    // segment decoder, one segment at a time
+                    uint32_t r0 = 0;
+                    while (r0 < cz.cnt) {
+                        const SegT sg = seg_from(cz, r0, cz.cnt);
+                        stage_seg(cur, cz, sg, 0);
+                        cp_async_commit();
+                        cp_async_wait<0>();
+                        __syncwarp();
+                        decode_seg(t, cur, cz, sg, 0);
+                        __syncwarp();
+                        r0 = sg.r1;
+                    }
+                } else {
+                    decode_partial(t, cur, cz);
+                }
+                __syncwarp();  // the region is restaged by the next tile
+                const uint64_t tnn = tile_of(__shfl_sync(0xffffffffu, iraw, 0));
+                t = tn;
+                cur = nx;
+                tn = tnn;
+                if (tn < p.nW) load_meta(tn, nx);
+            }
+        }
+    };
     auto nc_loop = [&]() {
         n_items = *p.n_nctile * split;
         uint32_t part, pn;
@@ -1418,7 +1632,11 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 8 && VPL == 4) ? 2 : SZX_DM
     // the split adapts to the field's fraction of nonconstant blocks.  (Decode
     // warps joining the fill as well, SZX_SWITCH = 3, measured slower: more
     // concurrent fill streams cut the write rate -- NYX density 107 -> 149 us.)
-    if (wid < C::FILLW) {
+    if (p.ts) {
+        ts_loop();
+        SZX_TL(2);
+        fill_ts();
+    } else if (wid < C::FILLW) {
         fill_loop();
         SZX_TL(2);
         if (SZX_SWITCH & 2) nc_loop();

@@ -467,17 +467,19 @@ __global__ void __launch_bounds__(32 * NW + 32, sizeof(T) == 4 ? SZX_EMINB : 3) 
     const int q = lane >> 3, ql = lane & 7;
     const int j = warp * 4 + q;  // this quarter's block within the tile
     // copy out tile kk (its offset produced by the scanner)
-    auto retire = [&](uint32_t kk) {
+    // pv: thread 0's early read of the tile's prefix word (issued an iteration
+    // earlier so its L2 latency overlaps the encode; re-polled if not yet written)
+    auto retire = [&](uint32_t kk, uint64_t pv) {
         const int sl = (int)(kk % NS);
         if (tid == 0) {
             SZX_ETL(s_tile[sl], 2);
-            uint64_t v;
             uint32_t ns = 32;
-            while (!((v = ld_relaxed(&p.prefix_e[s_tile[sl]])) >> 63)) {
+            while (!(pv >> 63)) {
                 __nanosleep(ns);
                 ns = ns < 256 ? 2 * ns : ns;
+                pv = ld_relaxed(&p.prefix_e[s_tile[sl]]);
             }
-            s_excl[sl] = v & ~(1ull << 63);
+            s_excl[sl] = pv & ~(1ull << 63);
         }
         bar_compute(C::NTC);
         copy_out_tile<C::NTC>(slot_addr(sl), out + off_pl + s_excl[sl], s_T[sl]);
@@ -534,6 +536,8 @@ __global__ void __launch_bounds__(32 * NW + 32, sizeof(T) == 4 ? SZX_EMINB : 3) 
                 asm volatile("st.shared.v4.u32 [%0], {%1,%1,%1,%1};" ::"r"(stg + 16u * c), "r"(0u) : "memory");
         }
         if (tid == 0) s_cur = atomicAdd(&p.ctr[3], 1u);  // the next tile (prefetched below)
+        uint64_t pv = 0;  // the prefix of the tile retired at the end of this iteration
+        if (tid == 0 && k + 1 >= NS) pv = ld_relaxed(&p.prefix_e[s_tile[(k + 1) % NS]]);
         const uint32_t wib = ib + (uint32_t)buf * C::IN + (uint32_t)warp * 4u * C::BW;  // this warp's 4 staged blocks
         const uint32_t mk = __shfl_sync(0xffffffffu, mc.mk, q);
         const T mu = TR::from(__shfl_sync(0xffffffffu, mc.mu, q));
@@ -651,13 +655,13 @@ __global__ void __launch_bounds__(32 * NW + 32, sizeof(T) == 4 ? SZX_EMINB : 3) 
         }
         // the next tile's values: its metadata arrived during the scan / pack
         if (nxt < ntiles) stage(mn, buf ^ 1);
-        if (k + 1 >= NS) retire(k + 1 - NS);  // (its barrier also orders this pack before the next zeroing)
+        if (k + 1 >= NS) retire(k + 1 - NS, pv);  // (its barrier also orders this pack before the next zeroing)
         cur = nxt;
         mc = mn;
     }
     // drain: the tiles still in their slots, in order
     const uint32_t k0 = k + 1 >= NS ? k + 1 - NS : 0;
-    for (uint32_t kk = k0; kk < k; kk++) retire(kk);
+    for (uint32_t kk = k0; kk < k; kk++) retire(kk, tid == 0 ? ld_relaxed(&p.prefix_e[s_tile[kk % NS]]) : 0);
 }
 
 }  // namespace szx
