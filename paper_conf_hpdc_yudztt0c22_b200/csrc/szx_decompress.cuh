@@ -200,6 +200,25 @@ __device__ inline void stage_u16(uint16_t* s_dst, const uint16_t* __restrict__ z
     }
 }
 
+// diagnostic timing builds only: index-phase stamps of thread 0 per index CTA
+// (after the first prefix, after the second prefix, after the per-tile pass)
+#ifndef SZX_TIMELINE
+#define SZX_TIMELINE 0
+#endif
+#if SZX_TIMELINE
+__device__ uint64_t g_tli[2048 * 4];
+#define SZX_TLI(k)                                                                    \
+    do {                                                                              \
+        if (threadIdx.x == 0 && blockIdx.x < 2048) {                                  \
+            uint64_t t_;                                                              \
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_) : : "memory");       \
+            g_tli[(uint64_t)blockIdx.x * 4 + (k)] = t_;                               \
+        }                                                                             \
+    } while (0)
+#else
+#define SZX_TLI(k) do { } while (0)
+#endif
+
 template <int W>
 __device__ inline void index_phase(const DPlan& p, const uint8_t* __restrict__ in, const DHdr& hd,
                                    uint16_t* s_zs, uint64_t* s_w) {
@@ -227,7 +246,9 @@ __device__ inline void index_phase(const DPlan& p, const uint8_t* __restrict__ i
         cnt += __popc(x) | (nc_tile(w, x) << 32);
     }
     const uint64_t aggP = cta_sum64(cnt, s_w);
+    SZX_TLI(0);
     const uint64_t exP = grid_excl_prefix(p.slot_a, p.res_a, &p.ctr[0], aggP, s_w, (uint32_t)G);
+    SZX_TLI(1);
     const uint64_t aggA = aggP & 0xFFFFFFFFu, exA = exP & 0xFFFFFFFFu;
     uint64_t runT = exP >> 32;
     const bool ok = exA + aggA <= hd.nnc;
@@ -245,7 +266,9 @@ __device__ inline void index_phase(const DPlan& p, const uint8_t* __restrict__ i
         }
     }
     const uint64_t aggZ = cta_sum64(zsum, s_w);
+    SZX_TLI(2);
     const uint64_t exZ = grid_excl_prefix(p.slot_z, p.res_z, &p.ctr[3], aggZ, s_w, (uint32_t)G);
+    SZX_TLI(3);
     // (3) per tile: ncpre and tbase
     uint64_t runA = exA, runZ = exZ;
     for (uint64_t wc = w0; wc < w1; wc += kIndexChunk) {
@@ -265,9 +288,24 @@ __device__ inline void index_phase(const DPlan& p, const uint8_t* __restrict__ i
             if (ok) stage_u16(s_zs, zs, runA, tot);
             __syncthreads();
         }
+        // per-tile payload bytes.  Dense tiles: the warp sums each of its 32
+        // tiles' zsizes together (consecutive u16 reads; a thread-serial loop
+        // over 32 zsizes per thread hits 2 banks from 32 threads)
         uint64_t sum = 0;
-        if (ok)
-            for (uint32_t j = 0; j < cw; j++) sum += s_zs[ex + j];
+        if (ok && (!SZX_IDXCOOP || __reduce_min_sync(0xffffffffu, cw) < 16u)) {
+            for (uint32_t j = 0; j < cw; j++) sum += s_zs[ex + j];  // a warp with a sparse tile: serial sums
+        } else if (ok) {
+            const int lane = threadIdx.x & 31;
+#pragma unroll 4
+            for (int k = 0; k < 32; k++) {
+                const uint32_t exk = __shfl_sync(0xffffffffu, (uint32_t)ex, k);
+                const uint32_t cwk = __shfl_sync(0xffffffffu, cw, k);
+                uint32_t v = (uint32_t)lane < cwk ? (uint32_t)s_zs[exk + lane] : 0u;
+#pragma unroll
+                for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+                if (lane == k) sum = v;
+            }
+        }
         uint64_t totz;
         const uint64_t exz = cta_scan256(sum, &totz, s_w);
         if (w < w1) p.tbase[w] = runZ + exz;
@@ -923,6 +961,9 @@ struct DecWCfg {
 #define SZX_SWITCH 2
 #endif
     static constexpr int FILLW = SZX_FILLW;         // fill warps per CTA (the rest decode)
+#ifndef SZX_IDXCOOP
+#define SZX_IDXCOOP 1    // index phase: warp-cooperative per-tile zsize sums on dense tiles
+#endif
 #ifndef SZX_TSUNC
 #define SZX_TSUNC 0  // thread-serial window: unpredicated look-ahead load (measured slower)
 #endif
@@ -945,9 +986,6 @@ struct DecWCfg {
 // Diagnostic timing builds only (-DSZX_TIMELINE=1, scripts/timeline.py): per
 // warp of k_decode_w, %globaltimer at kernel entry, index ready, fill done,
 // nonconstant tiles done.
-#ifndef SZX_TIMELINE
-#define SZX_TIMELINE 0
-#endif
 #if SZX_TIMELINE
 constexpr int kTlCtas = 2048;
 __device__ uint64_t g_tl[kTlCtas * 8 * 4];

@@ -437,6 +437,9 @@ __device__ inline uint64_t grid_excl_prefix(uint64_t* slots, uint64_t* res, uint
     return s_val;
 }
 
+#ifndef SZX_GBAR_NS
+#define SZX_GBAR_NS 256  // grid barrier: polling back-off cap (ns)
+#endif
 // Grid barrier: every global write made by any thread of any CTA before the
 // call is visible to every thread after it.  `ctr` must be zero.
 __device__ inline void grid_barrier(uint32_t* ctr) {
@@ -444,7 +447,11 @@ __device__ inline void grid_barrier(uint32_t* ctr) {
     if (threadIdx.x == 0) {
         __threadfence();
         atomicAdd(ctr, 1u);
-        while (ld_acquire_u32(ctr) < gridDim.x) __nanosleep(64);
+        uint32_t ns = 32;
+        while (ld_acquire_u32(ctr) < gridDim.x) {
+            __nanosleep(ns);
+            ns = ns < SZX_GBAR_NS ? 2 * ns : ns;
+        }
         __threadfence();
     }
     __syncthreads();

@@ -70,6 +70,16 @@ print(json.dumps({
     "decode_warps_done": q(dec[:, :, 3]),
     "kernel_span_us": round(float(us[:, :, 3].max()), 1),
 }))
+fi = L.szx_debug_timeline_index
+fi.argtypes = [ctypes.c_void_p, ctypes.c_uint64]
+bi = np.zeros(2048 * 4, dtype=np.uint64)
+assert fi(bi.ctypes.data, bi.size) == 0
+ti = bi.reshape(2048, 4).astype(np.int64)
+ti = ti[ti[:, 0] != 0]
+if ti.size:
+    ui = (ti - t0) / 1000.0
+    print(json.dumps({"index_ctas": int(ti.shape[0]), "local_counts_done": q(ui[:, 0]), "prefix1_done": q(ui[:, 1]),
+                      "zsize_sums_done": q(ui[:, 2]), "prefix2_done": q(ui[:, 3])}))
 if os.environ.get("DETAIL"):
     # index-ready time of warp 0 by CTA range (index CTAs first)
     for a in range(0, ctas, 37):
