@@ -180,6 +180,9 @@ __device__ inline uint64_t cta_scan256(uint64_t v, uint64_t* agg, uint64_t* s_w 
 #ifndef SZX_DQUARTER
 #define SZX_DQUARTER 0   // float32 b = 128: quarter-warp (1) or half-warp (0) block decoder
 #endif
+#ifndef SZX_IDXCOOP
+#define SZX_IDXCOOP 1    // index phase: warp-cooperative per-tile zsize sums on dense tiles
+#endif
 constexpr int kIndexChunk = 256;
 
 // Copy zs[i0, i0 + cnt) (cnt <= 32 * kIndexChunk) into shared memory with
@@ -961,9 +964,6 @@ struct DecWCfg {
 #define SZX_SWITCH 2
 #endif
     static constexpr int FILLW = SZX_FILLW;         // fill warps per CTA (the rest decode)
-#ifndef SZX_IDXCOOP
-#define SZX_IDXCOOP 1    // index phase: warp-cooperative per-tile zsize sums on dense tiles
-#endif
 #ifndef SZX_TSUNC
 #define SZX_TSUNC 0  // thread-serial window: unpredicated look-ahead load (measured slower)
 #endif
