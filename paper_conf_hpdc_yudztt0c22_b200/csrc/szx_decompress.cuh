@@ -1528,17 +1528,26 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 8 && VPL == 4) ? 2 : SZX_DM
     // staged, then decoded -- the warps of the SM hide each other's staging.
     auto ts_loop = [&]() {
         if constexpr (sizeof(T) == 4 && VPL == 4 && !QUAL) {
-            // software pipeline over tiles: at tile k the ticket of tile k+2 is
-            // in flight (atomic, then its list entry), the metadata of tile k+1
-            // is loaded and its zsizes are being read -- none of these global
-            // latencies is waited for inside the tile that issues them
-            n_items = *p.n_nctile;
-            auto tile_of = [&](uint32_t i) -> uint64_t { return i < n_items ? (uint64_t)p.nctile[i] : p.nW; };
-            uint32_t i0 = 0, i1 = 0;
-            if (lane == 0) { i0 = atomicAdd(&p.ctr[4], 1u); i1 = atomicAdd(&p.ctr[4], 1u); }
-            uint64_t t = tile_of(__shfl_sync(0xffffffffu, i0, 0));
-            uint64_t tn = tile_of(__shfl_sync(0xffffffffu, i1, 0));
-            TileMeta<U> cur, nx;
+            // Tickets are tile numbers (dense streams: nearly every tile holds
+            // nonconstant blocks; the rare all-constant ones are skipped), and
+            // the per-tile global reads are pipelined so that none is waited for
+            // in the iteration that issues it: at the top of tile k the ticket of
+            // tile k+2 is taken and the zsizes of tile k+1 requested (its
+            // metadata arrived during tile k-1), in the middle of tile k (after
+            // its staging is issued) the metadata of tile k+2 is requested.
+            auto ticket = [&]() -> uint32_t {
+                uint32_t v = 0;
+                if (lane == 0) v = atomicAdd(&p.ctr[4], 1u);
+                return v;
+            };
+            auto tile_of = [&](uint32_t raw) -> uint64_t {
+                const uint64_t v = p.t_lo + __shfl_sync(0xffffffffu, raw, 0);
+                return v < p.nWi ? v : p.nW;
+            };
+            const uint32_t r0 = ticket(), r1 = ticket();
+            uint64_t t = tile_of(r0);
+            uint64_t tn = tile_of(r1);
+            TileMeta<U> cur, nx, n2;
             if (t < p.nW) {
                 load_meta(t, cur);
                 load_zl(cur);
@@ -1546,12 +1555,20 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 8 && VPL == 4) ? 2 : SZX_DM
             if (tn < p.nW) load_meta(tn, nx);
             const uint32_t region = slot0, tb = region, sa = region + C::TS_TB;
             while (t < p.nW) {
-                uint32_t iraw = 0;  // the ticket of the tile after next (read at the end of this tile)
-                if (lane == 0) iraw = atomicAdd(&p.ctr[4], 1u);
-                const TileZ cz = tile_z(cur);
+                const uint32_t iraw = ticket();  // tile k+2 (resolved in the middle of this tile)
                 if (tn < p.nW) load_zl(nx);
+                const TileZ cz = tile_z(cur);
                 const uint64_t bytes = cur.end - cur.base;
-                if (!cz.ok) {
+                uint64_t tnn = p.nW;
+                bool asked = false;
+                auto ask_next = [&]() {  // the metadata of tile k+2
+                    tnn = tile_of(iraw);
+                    if (tnn < p.nW) load_meta(tnn, n2);
+                    asked = true;
+                };
+                if (t < nW_full && cur.word == 0u) {
+                    // all-constant tile (the fill writes it)
+                } else if (!cz.ok) {
                     if (lane == 0) set_corrupt(p.err);
                 } else if (t < nW_full && cz.cnt >= 24u && bytes + 15u <= (uint64_t)C::TS_STAGE) {
                     // stage the tile's payload (16-byte chunks), then decode a block per lane
@@ -1563,6 +1580,7 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 8 && VPL == 4) ? 2 : SZX_DM
                         cp_async16_zfill(sa + (uint32_t)(ga - gA), reinterpret_cast<const void*>(ga), rem < 16 ? (uint32_t)rem : 16u);
                     }
                     cp_async_commit();
+                    ask_next();
                     const uint32_t sbase = sa + (uint32_t)(g0 & 15);
                     const bool has = (cur.word >> lane) & 1u;
                     const uint32_t rank = __popc(cur.word & ((1u << lane) - 1u));
@@ -1596,11 +1614,11 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 8 && VPL == 4) ? 2 : SZX_DM
                     decode_partial(t, cur, cz);
                 }
                 __syncwarp();  // the region is restaged by the next tile
-                const uint64_t tnn = tile_of(__shfl_sync(0xffffffffu, iraw, 0));
+                if (!asked) ask_next();
                 t = tn;
                 cur = nx;
                 tn = tnn;
-                if (tn < p.nW) load_meta(tn, nx);
+                nx = n2;
             }
         }
     };

@@ -3,6 +3,7 @@ P:L2321-2336), the path dense float32 b = 128 streams of >= ~22 M values take
 (`DPlan::ts`, szx_api.cu).  The input mixes every tile shape that path meets:
 all-nonconstant tiles, tiles with 24-31 nonconstant blocks (thread-serial +
 constant fill), tiles with fewer (segment decoder inside the dense loop),
+all-constant tiles,
 raw blocks (a NaN forces R = 32, reading R14/R15) among thread-serial tiles,
 and a partial last block.  Stream bytes and reconstruction bits are compared
 with the oracle, the decoder is also run on the oracle's own bytes, and
@@ -33,6 +34,7 @@ def _mixed_dense(seed_field: int = 1, n_edge: int = 320, tail: int = 77) -> np.n
     t = np.arange(nW)
     blk[t % 7 == 3, :6, :] = 1.5e6           # 26 nonconstant blocks: thread-serial + constant fill
     blk[t % 11 == 5, :20, :] = -2.0e6        # 12 nonconstant blocks: segment decoder
+    blk[t % 17 == 8, :, :] = 0.25            # all-constant tiles (skipped by the dense loop, filled after)
     sel = np.nonzero(t % 13 == 1)[0]
     blk[sel, 5, 17] = np.nan                 # a raw block in an otherwise dense tile
     blk[sel[::3], 9, :] = np.inf             # an all-Inf block (raw: Inf radius, R14)
