@@ -1340,7 +1340,7 @@ int szx_debug_timeline(uint64_t* h_dst, uint64_t n) {
     const uint64_t cap = sizeof(szx::g_tl) / sizeof(uint64_t);
     return cudaMemcpyFromSymbol(h_dst, szx::g_tl, 8 * (n < cap ? n : cap)) == cudaSuccess ? SZX_OK : SZX_ECUDA;
 }
-// ... and the index-phase stamps of every index CTA (4 x u64 per CTA)
+// ... and the index-phase stamps of every CTA (8 x u64 per CTA)
 int szx_debug_timeline_index(uint64_t* h_dst, uint64_t n) {
     const uint64_t cap = sizeof(szx::g_tli) / sizeof(uint64_t);
     return cudaMemcpyFromSymbol(h_dst, szx::g_tli, 8 * (n < cap ? n : cap)) == cudaSuccess ? SZX_OK : SZX_ECUDA;

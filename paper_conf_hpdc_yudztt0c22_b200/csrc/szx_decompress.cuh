@@ -209,13 +209,13 @@ __device__ inline void stage_u16(uint16_t* s_dst, const uint16_t* __restrict__ z
 #define SZX_TIMELINE 0
 #endif
 #if SZX_TIMELINE
-__device__ uint64_t g_tli[2048 * 4];
+__device__ uint64_t g_tli[2048 * 8];
 #define SZX_TLI(k)                                                                    \
     do {                                                                              \
         if (threadIdx.x == 0 && blockIdx.x < 2048) {                                  \
             uint64_t t_;                                                              \
             asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_) : : "memory");       \
-            g_tli[(uint64_t)blockIdx.x * 4 + (k)] = t_;                               \
+            g_tli[(uint64_t)blockIdx.x * 8 + (k)] = t_;                               \
         }                                                                             \
     } while (0)
 #else
@@ -316,6 +316,7 @@ __device__ inline void index_phase(const DPlan& p, const uint8_t* __restrict__ i
         runZ += totz;
         __syncthreads();  // s_zs is refilled by the next chunk
     }
+    SZX_TLI(4);
     if (threadIdx.x == 0) {
         if (!ok) set_corrupt(p.err);
         if (c == G - 1) {
@@ -1132,6 +1133,7 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 8 && VPL == 4) ? 2 : SZX_DM
     // the barrier measured slower: their traffic stretches the latency-bound
     // index phase -- NYX velocity index 16 -> 22 us, Hurricane decode +8 us.)
     grid_barrier(&p.ctr[2]);
+    SZX_TLI(5);
     SZX_TL(1);
     const int lane = threadIdx.x & 31;
     const int wid = threadIdx.x >> 5;

@@ -49,6 +49,25 @@ x = synth.nyx_like(0, n=32).reshape(-1).cuda()
 mm = szx.local_minmax(x)
 e = (1e-3 * (mm[1] - mm[0])).reshape(1).contiguous()
 s = szx.compress_shard(x, 1e-3, e, "rel", 128)
+# the dense float32 decoder loop (thread-serial tiles; >= ~22 M values): mixed tile shapes,
+# a raw block and an all-constant tile, decoded once (SANITIZE_TS=0 skips it)
+if os.environ.get("SANITIZE_TS", "1") == "1":
+    xt = synth.nyx_like(1, n=288).reshape(-1).numpy().copy()[:-77]
+    nW = xt.size // 4096
+    blk = xt[: nW * 4096].reshape(nW, 32, 128)
+    blk[3::7, :6, :] = 1.5e6
+    blk[5::11, :20, :] = -2.0e6
+    blk[8::17, :, :] = 0.25
+    blk[1::13, 5, 17] = np.nan
+    s = szx.compress(torch.from_numpy(xt).cuda(), 1e-3, "rel", 128)
+    ref = oracle.compress(xt, 1e-3, oracle.REL, 128)
+    if s.cpu().numpy().tobytes() != ref.tobytes():
+        print("stream mismatch (dense)")
+        ok = False
+    y = szx.decompress(s)
+    if not np.array_equal(y.cpu().numpy().view(np.uint32), oracle.decompress(ref).view(np.uint32)):
+        print("reconstruction mismatch (dense)")
+        ok = False
 torch.cuda.synchronize()
 print("sanitize driver:", "ok" if ok else "MISMATCH")
 sys.exit(0 if ok else 1)

@@ -72,14 +72,18 @@ print(json.dumps({
 }))
 fi = L.szx_debug_timeline_index
 fi.argtypes = [ctypes.c_void_p, ctypes.c_uint64]
-bi = np.zeros(2048 * 4, dtype=np.uint64)
+bi = np.zeros(2048 * 8, dtype=np.uint64)
 assert fi(bi.ctypes.data, bi.size) == 0
-ti = bi.reshape(2048, 4).astype(np.int64)
-ti = ti[ti[:, 0] != 0]
+tall = bi.reshape(2048, 8).astype(np.int64)
+ti = tall[tall[:, 0] != 0]
 if ti.size:
     ui = (ti - t0) / 1000.0
     print(json.dumps({"index_ctas": int(ti.shape[0]), "local_counts_done": q(ui[:, 0]), "prefix1_done": q(ui[:, 1]),
-                      "zsize_sums_done": q(ui[:, 2]), "prefix2_done": q(ui[:, 3])}))
+                      "zsize_sums_done": q(ui[:, 2]), "prefix2_done": q(ui[:, 3]), "per_tile_pass_done": q(ui[:, 4])}))
+tb = tall[:ctas, 5]
+tb = tb[tb != 0]
+if tb.size:
+    print(json.dumps({"barrier_passed_all_ctas": q((tb - t0) / 1000.0)}))
 if os.environ.get("DETAIL"):
     # index-ready time of warp 0 by CTA range (index CTAs first)
     for a in range(0, ctas, 37):
