@@ -356,7 +356,7 @@ void enqueue_encode(const void* d_in, const Plan& p, const CLayout& L, uint8_t* 
     if constexpr (VPL == 4) {
         if (SZX_FUSED) {
             // b = 128: the fused encoder; float64 keeps 2 staging slots (smem)
-            constexpr int NS = sizeof(T) == 4 ? SZX_ENS : 2;
+            constexpr int NS = sizeof(T) == 4 ? SZX_ENS : SZX_ENS64;
             using EC = EncCfg<T, SZX_ENW, NS>;
             auto kern = k_encode_fused<T, SZX_ENW, NS>;
             const int occ_e = kernel_occupancy(kern, EC::SMEM, 1, EC::NT);

@@ -183,6 +183,9 @@ __device__ inline uint64_t cta_scan256(uint64_t v, uint64_t* agg, uint64_t* s_w 
 #ifndef SZX_IDXCOOP
 #define SZX_IDXCOOP 1    // index phase: warp-cooperative per-tile zsize sums on dense tiles
 #endif
+#ifndef SZX_DMINB64
+#define SZX_DMINB64 2    // float64 b = 128 decoder: CTAs per SM (register budget of the half-warp f64 form)
+#endif
 constexpr int kIndexChunk = 256;
 
 // Copy zs[i0, i0 + cnt) (cnt <= 32 * kIndexChunk) into shared memory with
@@ -1100,7 +1103,7 @@ struct TileMeta {
 };
 
 template <typename T, int VPL, bool QUAL = false>
-__global__ void __launch_bounds__(256, (sizeof(T) == 8 && VPL == 4) ? 2 : SZX_DMINB) k_decode_w(DPlan p, const uint8_t* __restrict__ in, T* __restrict__ y) {
+__global__ void __launch_bounds__(256, (sizeof(T) == 8 && VPL == 4) ? SZX_DMINB64 : SZX_DMINB) k_decode_w(DPlan p, const uint8_t* __restrict__ in, T* __restrict__ y) {
     using TR = Traits<T>;
     using U = typename TR::U;
     using C = DecWCfg<T, VPL>;

@@ -45,6 +45,12 @@ namespace szx {
 #ifndef SZX_ENS
 #define SZX_ENS 3     // staging slots per encoder CTA (tiles in flight)
 #endif
+#ifndef SZX_ENS64
+#define SZX_ENS64 2   // the same for float64 (shared memory)
+#endif
+#ifndef SZX_EMINB64
+#define SZX_EMINB64 3 // float64 encoder CTAs per SM (register budget)
+#endif
 
 // Diagnostic timing builds only (-DSZX_ETIMELINE=1, scripts/enc_timeline.py):
 // %globaltimer per tile at publish, prefix written, retire start / end.
@@ -425,7 +431,7 @@ __device__ __forceinline__ void bar_compute(int nthreads) {
 // without waiting, so the scanner always advances; the grid is co-resident
 // (cooperative launch), so the scanner's CTA runs.
 template <typename T, int NW, int NS>
-__global__ void __launch_bounds__(32 * NW + 32, sizeof(T) == 4 ? SZX_EMINB : 3) k_encode_fused(const T* __restrict__ x, Plan p,
+__global__ void __launch_bounds__(32 * NW + 32, sizeof(T) == 4 ? SZX_EMINB : SZX_EMINB64) k_encode_fused(const T* __restrict__ x, Plan p,
                                                                          uint8_t* __restrict__ out) {
     using C = EncCfg<T, NW, NS>;
     using TR = Traits<T>;
