@@ -968,6 +968,9 @@ struct DecWCfg {
 #define SZX_SWITCH 2
 #endif
     static constexpr int FILLW = SZX_FILLW;         // fill warps per CTA (the rest decode)
+#ifndef SZX_TSASM
+#define SZX_TSASM 1  // thread-serial window slide as one PTX block
+#endif
 #ifndef SZX_TSUNC
 #define SZX_TSUNC 0  // thread-serial window: unpredicated look-ahead load (measured slower)
 #endif
@@ -1055,7 +1058,23 @@ __device__ __forceinline__ bool ts_decode_f32(uint32_t a, uint32_t R, uint32_t z
                 prev = w;
                 o[i] = raw ? __uint_as_float(w) : __fadd_rn(__uint_as_float(w * ps), mu);  // step 5
                 pos += m8;
-#if SZX_TSUNC
+#if SZX_TSASM
+                // slide one word (m8 <= 32: at most one per value), in one PTX
+                // block so the predicated load lands in nx itself (no move of a
+                // just-loaded register)
+                asm volatile(
+                    "{\n\t.reg .pred q;\n\t.reg .u32 ad;\n\t"
+                    "setp.ge.u32 q, %4, %3;\n\t"
+                    "@q add.u32 %3, %3, 32;\n\t"
+                    "@q mov.b32 %0, %1;\n\t"
+                    "@q mov.b32 %1, %2;\n\t"
+                    "shr.u32 ad, %3, 3;\n\t"
+                    "add.u32 ad, ad, %5;\n\t"
+                    "@q ld.shared.u32 %2, [ad];\n\t}"
+                    : "+r"(lo), "+r"(hi), "+r"(nx), "+r"(lim)
+                    : "r"(pos), "r"(wp8 - 4u)
+                    : "memory");
+#elif SZX_TSUNC
                 // slide one word (m8 <= 32: at most one per value); nx is re-read
                 // every value (unpredicated: no move of a just-loaded register)
                 const bool sl = pos >= lim;
