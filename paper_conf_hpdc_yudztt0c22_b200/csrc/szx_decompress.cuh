@@ -186,6 +186,12 @@ __device__ inline uint64_t cta_scan256(uint64_t v, uint64_t* agg, uint64_t* s_w 
 #ifndef SZX_DMINB64
 #define SZX_DMINB64 2    // float64 b = 128 decoder: CTAs per SM (register budget of the half-warp f64 form)
 #endif
+#ifndef SZX_IDXRED
+#define SZX_IDXRED 1           // index phase: redundant bitmap prefix instead of the first grid prefix
+#endif
+#ifndef SZX_IDXRED_MAXW
+#define SZX_IDXRED_MAXW 4096   // ... for bitmaps up to this many 32-block words (16 KB; larger: measured slower)
+#endif
 constexpr int kIndexChunk = 256;
 
 // Copy zs[i0, i0 + cnt) (cnt <= 32 * kIndexChunk) into shared memory with
@@ -246,14 +252,37 @@ __device__ inline void index_phase(const DPlan& p, const uint8_t* __restrict__ i
     // (1) nonconstant blocks (low 32 bits) and such tiles (high 32 bits) in the
     // range -> starting nonconstant index and list position.  Both fit 32 bits:
     // nB <= kMaxN / 32 = 2^31 (static_assert beside kMaxN in szx_api.cu).
-    uint64_t cnt = 0;
-    for (uint64_t w = w0 + threadIdx.x; w < w1; w += kIndexChunk) {
-        const uint32_t x = word_at(w);
-        cnt += __popc(x) | (nc_tile(w, x) << 32);
+    // Bitmaps up to SZX_IDXRED_MAXW words: every index CTA also counts the
+    // words before its range itself (16-byte loads, mostly L2 hits), which
+    // replaces the first grid-wide prefix; larger ones take the prefix.
+    const bool red = SZX_IDXRED && p.nWi <= (uint64_t)SZX_IDXRED_MAXW;
+    uint64_t cnt = 0, pre = 0;
+    if (red) {
+        const uint64_t nq = (w1 + 3) / 4;  // 4-word groups of [0, w1) (the bitmap section is 16-byte padded)
+#pragma unroll 8
+        for (uint64_t qq = threadIdx.x; qq < nq; qq += kIndexChunk) {
+            const uint4 v = *reinterpret_cast<const uint4*>(bm + 4 * qq);
+            const uint32_t e[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+            for (int k = 0; k < 4; k++) {
+                const uint64_t w = 4 * qq + k;
+                uint32_t x = e[k];
+                if (w == p.nW - 1 && (p.nB & 31)) x &= (1u << (p.nB & 31)) - 1u;
+                const uint64_t a = w < w1 ? (__popc(x) | (nc_tile(w, x) << 32)) : 0u;
+                if (w < w0) pre += a;
+                else cnt += a;
+            }
+        }
+    } else {
+        for (uint64_t w = w0 + threadIdx.x; w < w1; w += kIndexChunk) {
+            const uint32_t x = word_at(w);
+            cnt += __popc(x) | (nc_tile(w, x) << 32);
+        }
     }
     const uint64_t aggP = cta_sum64(cnt, s_w);
     SZX_TLI(0);
-    const uint64_t exP = grid_excl_prefix(p.slot_a, p.res_a, &p.ctr[0], aggP, s_w, (uint32_t)G);
+    const uint64_t exP = red ? cta_sum64(pre, s_w)
+                             : grid_excl_prefix(p.slot_a, p.res_a, &p.ctr[0], aggP, s_w, (uint32_t)G);
     SZX_TLI(1);
     const uint64_t aggA = aggP & 0xFFFFFFFFu, exA = exP & 0xFFFFFFFFu;
     uint64_t runT = exP >> 32;
