@@ -396,17 +396,40 @@ def main():
     kern_per_step = szx.launch_count() - l1
     gpu_launches = kern_per_step * a.steps if graph is not None else launches_eager
 
-    # ---- phase breakdown (eager, events between phases; median over steps)
+    # ---- phase breakdown: each field's compress and decompress captured in their
+    # own CUDA graphs (as the step runs them; eager launches with --no-graph),
+    # events between the phases, median over repetitions
     kb = max(5, min(a.steps, 30))
+    pg = None
+    if graph is not None:
+        try:
+            pg = []
+            for i in range(len(xs)):
+                gc, gd = torch.cuda.CUDAGraph(), torch.cuda.CUDAGraph()
+                with torch.cuda.graph(gc, stream=stream):
+                    compress_f(i)
+                with torch.cuda.graph(gd, stream=stream):
+                    decompress_f(i)
+                pg.append((gc, gd))
+        except Exception as ex:  # noqa: BLE001
+            print(f"# phase graph capture failed ({type(ex).__name__}: {ex}); eager phases", file=sys.stderr)
+            pg = None
+            torch.cuda.synchronize()
     ph = {i: ([], []) for i in range(len(xs))}
     with torch.cuda.stream(stream):
         for _ in range(kb):
             for i in range(len(xs)):
                 e0, e1, e2 = (torch.cuda.Event(enable_timing=True) for _ in range(3))
                 e0.record()
-                compress_f(i)
+                if pg is not None:
+                    pg[i][0].replay()
+                else:
+                    compress_f(i)
                 e1.record()
-                decompress_f(i)
+                if pg is not None:
+                    pg[i][1].replay()
+                else:
+                    decompress_f(i)
                 e2.record()
                 ph[i][0].append((e0, e1))
                 ph[i][1].append((e1, e2))
@@ -550,7 +573,8 @@ def main():
             "gpu_launches": gpu_launches, "kernels_per_step": kern_per_step, "graph": graph is not None,
             "clocks": clocks,
             "timing": "value/ms_per_step: CUDA events around K replays of the step's CUDA graph (eager if "
-                      "graph=false); fields.*: phase events in a separate eager pass; kernels_ms_per_launch / "
+                      "graph=false); fields.*: events around each field's compress / decompress CUDA graph (eager with --no-graph), "
+                      "median of the repetitions; kernels_ms_per_launch / "
                       "roofline: library CUDA events around each launch in a third pass",
             "paper_context": "cuSZx A100: 150-216 GB/s compress, 150-291 GB/s decompress (P:L3207-3220)",
         }
