@@ -153,6 +153,21 @@ def _ncu_kernel(summ, field: str, kernel: str):
     return None
 
 
+def _sm_count() -> int:
+    try:
+        import torch
+        return torch.cuda.get_device_properties(0).multi_processor_count
+    except Exception:  # noqa: BLE001
+        return 148
+
+
+def _sm_max_mhz() -> float:
+    try:
+        return float(json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["sm_max_mhz"])
+    except Exception:  # noqa: BLE001
+        return 1965.0
+
+
 def _peaks():
     try:
         return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"], "measured"
@@ -547,6 +562,14 @@ def main():
                                 "traffic": nv.get("dram_bytes") if nv else None,
                                 "traffic_source": summ_src if nv else None,
                                 "alg_bytes_per_launch": alg.get(dom), "ms_per_launch": kms[dom]}
+                if nv and nv.get("inst_executed"):
+                    # the same launch against the SM issue rate (warp-instructions from the
+                    # committed ncu capture of this field / live launch time; peak: 4 schedulers
+                    # x SMs x max clock, one warp-instruction per scheduler per cycle)
+                    ipeak = 4.0 * _sm_count() * _sm_max_mhz() * 1e6
+                    iach = nv["inst_executed"] / (kms[dom] / 1e3)
+                    roofs[fname]["issue"] = {"achieved": iach, "peak": ipeak, "unit": "warp-inst/s",
+                                             "frac": iach / ipeak, "source": summ_src}
                 tot = sum(kms.values())
                 if kms[dom] > dom_t:
                     dom_all, dom_t = (fname, dom), kms[dom]
