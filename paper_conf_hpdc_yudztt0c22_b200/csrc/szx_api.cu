@@ -186,7 +186,7 @@ CLayout clayout(uint64_t n, int W, uint32_t b) {
     L.nTC = cdiv(cdiv(L.nB, kWriteTile), 256);  // k_zscan CTAs (look-back status words)
     L.off_keys = 0;
     L.off_zero = 16;
-    L.nTE = cdiv(L.nB, 4 * SZX_ENW) + 1;  // k_encode_f32 tiles (look-back status words)
+    L.nTE = cdiv(L.nB, 4 * SZX_ENW) + 1;  // k_encode_fused tiles (scanner status words)
     L.zero_bytes = al16(16 + 16 * L.nTB + 8 * L.nTC + 16 * L.nTE);  // classify: 2 words per tile
     L.off_scal = L.off_zero + L.zero_bytes;
     L.off_stats = L.off_scal + 32;

@@ -1,30 +1,31 @@
-// szx_encode.cuh -- fused single-pass encoder for float32, b = 128 (sm_100a).
+// szx_encode.cuh -- the fused single-pass encoder for b = 128 (float32 and
+// float64, sm_100a): k_encode_fused.
 //
-//   k_encode_f32 (K2+K3+K4 in one pass over the nonconstant blocks)
-//
-// One read of the nonconstant blocks' values, one write of the payload: per
-// tile of 32 nonconstant blocks (the compacted list of k_classify, in block
-// order) a 256-thread CTA
-//   (1) stages the tile's 32 x 512 B with cp.async (prefetched one tile ahead,
-//       16-byte chunks swizzled so the quarter-warp reads are bank-conflict
-//       free);
-//   (2) encodes every block with a quarter-warp (8 lanes x 16 values): v_i =
-//       d_i - mu (Alg. 1 l.10), Formula 5's shift folded into the lead-byte
-//       count, 2-bit codes min(3, identical leading bytes) against the previous
-//       value (Sec. 6.1 steps 1-4; u_{-1} = 0, reading R6), mid-byte
+// One read of the nonconstant blocks' values, one write of the payload.  A CTA
+// of NW = 4 compute warps + 1 extra warp works on tiles of 4 x NW = 16
+// consecutive entries of k_classify's compacted nonconstant list (tickets in
+// order, the next ticket and its metadata prefetched):
+//   (1) each warp stages its 4 blocks with cp.async (16-byte chunks swizzled
+//       so the quarter-warp reads are bank-conflict free), the next tile's
+//       values while the current one is packed;
+//   (2) a quarter-warp (8 lanes x 16 values) encodes a block: v_i = d_i - mu
+//       (Alg. 1 l.10), Formula 5's shift folded into the lead-byte count, 2-bit
+//       codes min(3, identical leading bytes) against the previous value
+//       (Sec. 6.1 steps 1-4; u_{-1} = 0, reading R6), mid-byte
 //       counts, z_k = 1 + 32 + sum m_i;
-//   (3) scans the tile's z_k (warp 0) and publishes the tile's payload bytes for
-//       the decoupled look-back (the device-wide exclusive scan of block sizes,
-//       P:L2350-2377; 256 predecessors per round trip), warp 0 resolving it
-//       while the other warps pack;
-//   (4) packs [R][codes][mid-bytes] of every block into a zeroed shared-memory
-//       tile with OR reductions (reading R7/R8);
-//   (5) resolves the tile's payload offset and copies the tile out with
-//       16-byte stores, realigned to the output.
+//   (3) every warp scans the tile's 16 z_k; warp 0 writes the zsize entries and
+//       publishes the tile's payload bytes in its status word;
+//   (4) the quarter packs [R][codes][mid-bytes] into a zeroed shared-memory
+//       slot (one of NS = 3) with OR reductions (readings R7/R8);
+//   (5) the grid's tile scanner -- the extra warp of CTA 0 -- walks the status
+//       words in tile order and writes every tile's exclusive payload offset
+//       as soon as it and its predecessors have published (the device-wide
+//       exclusive scan of block sizes); tile k is copied out NS - 1
+//       tiles later with 16-byte stores realigned to its offset.
 // The R2 guard runs where k_classify could not prove it away (whole-warp
-// check, DESIGN.md s.3); raw blocks (R = 32) and the partial last block take a
-// whole-warp generic path.  Byte-identical to the three-pass encoder and the
-// oracle.
+// check, DESIGN.md s.3); raw blocks (R = full width) and the partial last block
+// take a whole-warp generic path.  Byte-identical to the three-pass encoder
+// (b != 128) and the oracle.
 #pragma once
 
 #include <type_traits>
@@ -78,68 +79,6 @@ __device__ __forceinline__ uint32_t swz16(uint32_t c) { return (c & ~7u) | ((c ^
 // the same for CPL chunks per quarter lane (4: float32, 8: float64)
 template <int CPL>
 __device__ __forceinline__ uint32_t swzc(uint32_t c) { return (c & ~7u) | ((c ^ (c / CPL)) & 7u); }
-
-// Decoupled look-back with a 256-entry window (8 status words per lane): the
-// exclusive prefix of `agg` over tiles [0, tile).  Tile `tile` must already
-// have published its aggregate (lb_publish).  All 32 lanes of one warp.
-__device__ inline void lb_publish(uint64_t* status, uint64_t tile, uint64_t agg) {
-    st_relaxed(&status[tile], (tile == 0 ? kFlagIncl : kFlagAgg) | agg);
-}
-__device__ inline uint64_t lb_resolve(uint64_t* status, uint64_t tile, uint64_t agg) {
-    constexpr int K = 8;  // status words per lane: a 256-tile window per round trip
-    if (tile == 0) return 0;
-    const int lane = threadIdx.x & 31;
-    uint64_t excl = 0;
-    int64_t base = (int64_t)tile - 1;
-    while (true) {
-        uint64_t st[K];
-#pragma unroll
-        for (int k = 0; k < K; k++) {
-            const int64_t idx = base - K * lane - k;
-            st[k] = idx >= 0 ? ld_relaxed(&status[idx]) : (kFlagIncl | 0);
-        }
-        int kf = K;      // nearest inclusive entry of this lane
-        int kv = K;      // nearest unpublished entry of this lane
-#pragma unroll
-        for (int k = K - 1; k >= 0; k--) {
-            if ((st[k] >> 62) == 2) kf = k;
-            if ((st[k] >> 62) == 0) kv = k;
-        }
-        const uint32_t pm = __ballot_sync(0xffffffffu, kf < K);
-        const int fl = pm ? __ffs(pm) - 1 : 32;            // lane holding the nearest inclusive
-        const int kfl = __shfl_sync(0xffffffffu, kf, fl & 31);
-        // every entry before the nearest inclusive one must be published
-        const bool need_ok = lane < fl ? kv == K : (lane == fl ? kv > kfl : true);
-        if (!__all_sync(0xffffffffu, need_ok)) {
-            // a predecessor has not published yet: one lane polls the nearest such entry
-            // (cheap on L2) before the window is read again
-            const uint32_t um = __ballot_sync(0xffffffffu, kv < K);
-            const int ul = __ffs(um) - 1;
-            const int kvl = __shfl_sync(0xffffffffu, kv, ul);
-            if (lane == 0) {
-                const uint64_t* w = &status[base - K * ul - kvl];
-                uint32_t ns = 64;
-                while (ld_relaxed(w) == 0) {
-                    __nanosleep(ns);
-                    ns = ns < 1024 ? 2 * ns : ns;
-                }
-            }
-            __syncwarp();
-            continue;
-        }
-        uint64_t v = 0;
-#pragma unroll
-        for (int k = 0; k < K; k++) {
-            const bool take = lane < fl || (lane == fl && k <= kfl);
-            v += take ? (st[k] & kValueMask) : 0;
-        }
-        excl += warp_sum64(v);
-        if (pm) break;
-        base -= 32 * K;
-    }
-    if (lane == 0) st_relaxed(&status[tile], kFlagIncl | (excl + agg));
-    return excl;
-}
 
 // Forward scanner of tile sizes (one warp for the whole grid): walks the
 // status array in tile order, 512 tiles per round trip, and writes every
