@@ -29,6 +29,7 @@
 #pragma once
 
 #include <type_traits>
+#include <utility>
 
 #include "szx_compress.cuh"
 
@@ -39,6 +40,9 @@ namespace szx {
 #endif
 #ifndef SZX_ERED3
 #define SZX_ERED3 1
+#endif
+#ifndef SZX_M8PACK
+#define SZX_M8PACK 1  // mid-byte counts packed 4 per register (no spill)
 #endif
 #ifndef SZX_ENW
 #define SZX_ENW 4     // compute warps per encoder CTA (tile = 4 x warps nonconstant blocks)
@@ -157,6 +161,32 @@ __device__ inline void tile_scanner(const uint64_t* status, uint64_t* prefix, ui
     }
 }
 
+// Per-value mid-byte counts (8 x m, <= 64) of a quarter lane's 16 values, one
+// byte each in 4 words (16 separate registers spilled to local memory at 72
+// registers per thread, the per-SMSP limit of 5 CTAs x 5 warps)
+struct M8 {
+#if SZX_M8PACK
+    uint32_t w[4];
+    template <int I>
+    __device__ __forceinline__ void set(uint32_t v) {
+        w[I >> 2] = (I & 3) ? (w[I >> 2] | (v << (8 * (I & 3)))) : v;
+    }
+    template <int I>
+    __device__ __forceinline__ uint32_t get() const { return __byte_perm(w[I >> 2], 0u, 0x4440u | (I & 3)); }
+#else
+    uint32_t w[16];
+    template <int I>
+    __device__ __forceinline__ void set(uint32_t v) { w[I] = v; }
+    template <int I>
+    __device__ __forceinline__ uint32_t get() const { return w[I]; }
+#endif
+};
+template <int... Is, typename F>
+__device__ __forceinline__ void unroll_impl(F&& f, std::integer_sequence<int, Is...>) { (f(std::integral_constant<int, Is>{}), ...); }
+// f(integral_constant<int, i>) for i = 0 .. N-1, in order (compile-time indices)
+template <int N, typename F>
+__device__ __forceinline__ void unroll(F&& f) { unroll_impl(f, std::make_integer_sequence<int, N>{}); }
+
 // ---- quarter-warp block encoder (full float32 block, 9 <= R < 32)
 struct QEnc {
     uint32_t v[16];     // normalised words bits(d_i - mu)
@@ -169,7 +199,7 @@ struct QEnc {
 // logical shift adds s identical leading zeros to both words; OR-ing 0xFF << s
 // into the XOR caps the count at 3.
 __device__ __forceinline__ void quarter_encode_f32(const float (&x)[16], float mu, uint32_t R, QEnc& e,
-                                                   uint32_t (&m8)[16]) {
+                                                   M8& m8) {
     const int ql = threadIdx.x & 7;
     const uint32_t s = (8u - (R & 7u)) & 7u;
     const uint32_t req = (R + s) >> 3;
@@ -179,22 +209,22 @@ __device__ __forceinline__ void quarter_encode_f32(const float (&x)[16], float m
     uint32_t prev = __shfl_up_sync(0xffffffffu, e.v[15], 1, 8);
     prev = ql == 0 ? 0u : prev;
     uint32_t codes = 0, msum = 0;
-#pragma unroll
-    for (int i = 0; i < 16; i++) {
+    unroll<16>([&](auto I) {
+        constexpr int i = decltype(I)::value;
         const uint32_t L = ((uint32_t)__clz((e.v[i] ^ prev) | cap) + s) >> 3;
         prev = e.v[i];
         codes |= L << (2 * i);
         const uint32_t m = req - umin(L, req);
-        m8[i] = 8u * m;
+        m8.template set<i>(8u * m);
         msum += m;
-    }
+    });
     e.codes = codes;
     e.msum = msum;
 }
 
 // Pack the quarter's block at shared byte address dst: [R][32 code bytes][mid-bytes];
 // mexcl = this lane's exclusive mid-byte offset within the block.
-__device__ __forceinline__ void quarter_pack_f32(const QEnc& e, const uint32_t (&m8)[16], uint32_t R,
+__device__ __forceinline__ void quarter_pack_f32(const QEnc& e, const M8& m8, uint32_t R,
                                                  uint32_t mexcl, uint32_t dst) {
     const int ql = threadIdx.x & 7;
     if (ql == 0) red_or_s(dst & ~3u, R << (8u * (dst & 3u)));
@@ -205,9 +235,9 @@ __device__ __forceinline__ void quarter_pack_f32(const QEnc& e, const uint32_t (
     }
     const uint32_t rs = 32u - R;     // v >> rs = the R kept bits (u >> drop)
     uint32_t a = dst + 33u + mexcl;
-#pragma unroll
-    for (int h = 0; h < 8; h++) {
-        const uint32_t n0 = m8[2 * h], n1 = m8[2 * h + 1];
+    unroll<8>([&](auto H) {
+        constexpr int h = decltype(H)::value;
+        const uint32_t n0 = m8.template get<2 * h>(), n1 = m8.template get<2 * h + 1>();
         // the mid-bytes: the low m_i bytes of the kept bits (bytes [W-req, W-L) of u)
         const uint32_t c0 = (e.v[2 * h] >> rs) & ~__funnelshift_lc(0u, 0xFFFFFFFFu, n0);
         const uint32_t c1 = (e.v[2 * h + 1] >> rs) & ~__funnelshift_lc(0u, 0xFFFFFFFFu, n1);
@@ -222,7 +252,7 @@ __device__ __forceinline__ void quarter_pack_f32(const QEnc& e, const uint32_t (
         red_or_nz(wa + 8u, __funnelshift_l(hi, 0u, sh));
 #endif
         a += (n0 + n1) >> 3;
-    }
+    });
 }
 
 // ---- the same for float64 blocks of b = 128 (8 lanes x 16 doubles): the lead
@@ -234,7 +264,7 @@ struct QEnc64 {
     uint32_t msum;
 };
 __device__ __forceinline__ void quarter_encode_f64(const double (&x)[16], double mu, uint32_t R, QEnc64& e,
-                                                   uint32_t (&m8)[16]) {
+                                                   M8& m8) {
     const int ql = threadIdx.x & 7;
     const uint32_t s = (8u - (R & 7u)) & 7u;
     const uint32_t req = (R + s) >> 3;  // 2 .. 8
@@ -244,20 +274,20 @@ __device__ __forceinline__ void quarter_encode_f64(const double (&x)[16], double
     uint32_t prevh = __shfl_up_sync(0xffffffffu, (uint32_t)(e.v[15] >> 32), 1, 8);
     prevh = ql == 0 ? 0u : prevh;
     uint32_t codes = 0, msum = 0;
-#pragma unroll
-    for (int i = 0; i < 16; i++) {
+    unroll<16>([&](auto I) {
+        constexpr int i = decltype(I)::value;
         const uint32_t h = (uint32_t)(e.v[i] >> 32);
         const uint32_t L = ((uint32_t)__clz((h ^ prevh) | cap) + s) >> 3;
         prevh = h;
         codes |= L << (2 * i);
         const uint32_t m = req - umin(L, req);
-        m8[i] = 8u * m;  // 0 .. 64
+        m8.template set<i>(8u * m);  // 0 .. 64
         msum += m;
-    }
+    });
     e.codes = codes;
     e.msum = msum;
 }
-__device__ __forceinline__ void quarter_pack_f64(const QEnc64& e, const uint32_t (&m8)[16], uint32_t R,
+__device__ __forceinline__ void quarter_pack_f64(const QEnc64& e, const M8& m8, uint32_t R,
                                                  uint32_t mexcl, uint32_t dst) {
     const int ql = threadIdx.x & 7;
     if (ql == 0) red_or_s(dst & ~3u, R << (8u * (dst & 3u)));
@@ -268,9 +298,9 @@ __device__ __forceinline__ void quarter_pack_f64(const QEnc64& e, const uint32_t
     }
     const uint32_t rs = 64u - R;  // v >> rs = the R kept bits
     uint32_t a = dst + 33u + mexcl;
-#pragma unroll
-    for (int i = 0; i < 16; i++) {
-        const uint32_t n = m8[i];
+    unroll<16>([&](auto I) {
+        constexpr int i = decltype(I)::value;
+        const uint32_t n = m8.template get<i>();
         // the low m_i bytes of the kept bits, as (lo, hi) words
         const uint64_t k = e.v[i] >> rs;
         const uint64_t c = n >= 64u ? k : (k & ((1ull << n) - 1ull));
@@ -280,7 +310,7 @@ __device__ __forceinline__ void quarter_pack_f64(const QEnc64& e, const uint32_t
         red_or_s(wa + 4u, __funnelshift_l(lo, hi, sh));
         red_or_s(wa + 8u, __funnelshift_l(hi, 0u, sh));
         a += n >> 3;
-    }
+    });
 }
 
 template <int O>
@@ -508,7 +538,7 @@ __global__ void __launch_bounds__(32 * NW + 32, sizeof(T) == 4 ? SZX_EMINB : SZX
         }
         const bool fast = !__any_sync(0xffffffffu, valid && (!full || R >= (uint32_t)TR::kFull));
         typename std::conditional<sizeof(T) == 4, QEnc, QEnc64>::type e;
-        uint32_t m8[16];
+        M8 m8;
         uint32_t mexcl = 0;
         uint32_t zex = 0;   // lane b < TILE: in-tile payload offset of block b
         uint32_t rfin = 0;  // generic path: the final R of block kq in byte kq (after the R2 guard)
