@@ -1346,6 +1346,12 @@ int szx_debug_timeline_index(uint64_t* h_dst, uint64_t n) {
     return cudaMemcpyFromSymbol(h_dst, szx::g_tli, 8 * (n < cap ? n : cap)) == cudaSuccess ? SZX_OK : SZX_ECUDA;
 }
 #endif
+#if SZX_GUARDSTAT
+// diagnostic builds only: {guarded blocks, warp-tiles} counted by the fused encoder since load
+int szx_debug_guardstat(uint64_t* h_dst) {
+    return cudaMemcpyFromSymbol(h_dst, szx::g_guardstat, 16) == cudaSuccess ? SZX_OK : SZX_ECUDA;
+}
+#endif
 #if SZX_ETIMELINE
 // diagnostic timing builds only: the fused encoder's per-tile timeline (4 x u64 per tile)
 int szx_debug_enc_timeline(uint64_t* h_dst, uint64_t n) {

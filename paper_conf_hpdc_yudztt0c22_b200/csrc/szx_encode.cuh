@@ -76,6 +76,13 @@ __device__ inline uint64_t gtimer() {
 #define SZX_ETL(tile, k) do { } while (0)
 #endif
 
+#ifndef SZX_GUARDSTAT
+#define SZX_GUARDSTAT 0  // diagnostic builds: count blocks whose R2 guard runs in the fused encoder
+#endif
+#if SZX_GUARDSTAT
+__device__ unsigned long long g_guardstat[2];
+#endif
+
 // 16-byte chunk c (0..31) of a staged block sits at swz16(c): lane ql of a
 // quarter reads chunks 4 ql .. 4 ql + 3, and the 8 lanes of one LDS.128 phase
 // then hit 8 distinct 16-byte bank groups
@@ -525,6 +532,12 @@ __global__ void __launch_bounds__(32 * NW + 32, sizeof(T) == 4 ? SZX_EMINB : SZX
         {   // R2 guard where classify could not prove it away: whole warp, one block at a time
             const bool ng = valid && full && !(rec & 0x80u) && R < (uint32_t)TR::kFull;
             uint32_t gm = __ballot_sync(0xffffffffu, ng && ql == 0);
+#if SZX_GUARDSTAT
+            if (lane == 0) {
+                atomicAdd(&g_guardstat[0], (unsigned long long)__popc(gm));
+                atomicAdd(&g_guardstat[1], 1ull);
+            }
+#endif
             while (gm) {
                 const int gl = __ffs(gm) - 1;
                 gm &= gm - 1;
