@@ -1067,10 +1067,15 @@ __device__ __forceinline__ bool ts_decode_f32(uint32_t a, uint32_t R, uint32_t z
     uint32_t pos = pos0, lim = 32u, prev = 0;
     const uint32_t wp8 = wp + 8u;
     const uint32_t sw = ((uint32_t)lane >> 2) & 1u;     // transpose swizzle (bank-conflict free)
+    // the lead codes: group g's 4 code bytes start at a + 1 + 4 g; the aligned
+    // words cw0 (this group's first) and cw1 (next) are loaded a group ahead
+    const uint32_t cb0 = (a + 1u) & ~3u, csh = 8u * (a + 1u);
+    uint32_t cw0 = lds_u32(cb0), cw1 = lds_u32(cb0 + 4u);
 #pragma unroll 1
     for (int g = 0; g < 8; g++) {
-        const uint32_t cb = a + 1u + 4u * (uint32_t)g;  // this group's 16 lead codes (4 bytes)
-        uint32_t cw = __funnelshift_r(lds_u32(cb & ~3u), lds_u32((cb & ~3u) + 4), 8u * cb);
+        uint32_t cw = __funnelshift_r(cw0, cw1, csh);  // this group's 16 lead codes
+        cw0 = cw1;
+        cw1 = lds_u32(cb0 + 8u + 4u * (uint32_t)g);    // (read past the codes on the last group: inside the payload / pad)
         cw ^= cw & (cw >> 1) & fix;
 #pragma unroll
         for (int h = 0; h < 2; h++) {
