@@ -997,6 +997,12 @@ struct DecWCfg {
 #define SZX_SWITCH 2
 #endif
     static constexpr int FILLW = SZX_FILLW;         // fill warps per CTA (the rest decode)
+#ifndef SZX_TSFL16
+#define SZX_TSFL16 1   // thread-serial decoder: transpose 16 values per flush (64-byte block segments)
+#endif
+#ifndef SZX_TSCLAMP
+#define SZX_TSCLAMP 1  // thread-serial decoder: payload reads clamped to the warp's region (no over-read pad)
+#endif
 #ifndef SZX_TSASM
 #define SZX_TSASM 1  // thread-serial window slide as one PTX block
 #endif
@@ -1012,8 +1018,9 @@ struct DecWCfg {
     // per-warp shared region: the two staging slots of the segment decoder, or
     // (thread-serial tiles) a 1 KB transpose buffer + one staging area + over-read pad
     static constexpr int REGION = SZX_DREGION > 2 * SLOT_ALLOC ? SZX_DREGION : 2 * SLOT_ALLOC;
-    static constexpr int TS_TB = 1024;               // transpose buffer: 32 blocks x 8 values
-    static constexpr int TS_PAD = 576;               // > 12 + 128 x 4 bytes a corrupt lane may over-read
+    static constexpr int TS_TB = SZX_TSFL16 ? 2048 : 1024;  // transpose buffer: 32 blocks x 16 (8) values
+    static constexpr int TS_PAD = SZX_TSCLAMP ? 16 : 576;   // reads clamped to the region, or > 12 + 128 x 4
+                                                            // bytes a corrupt lane may over-read
     static constexpr int TS_STAGE = REGION - TS_TB - TS_PAD;
     static constexpr int SMEM = NWARP * REGION;
     static_assert(SMEM >= kIndexChunk * 32 * 2, "index-phase scratch aliases the slots");
@@ -1052,7 +1059,10 @@ __device__ uint64_t g_tl[kTlCtas * 8 * 4];
 // store nothing).  Returns false (this lane) on a size mismatch.
 template <bool RAWOK>
 __device__ __forceinline__ bool ts_decode_f32(uint32_t a, uint32_t R, uint32_t zz, float mu, uint32_t tb,
-                                              float* __restrict__ yt, uint32_t word) {
+                                              float* __restrict__ yt, uint32_t word, uint32_t lastw) {
+    // SZX_TSCLAMP: every payload read is clamped to lastw (the region's last
+    // word), so a corrupt lane cannot leave its warp's region without a pad
+    auto ldc = [&](uint32_t ad) -> uint32_t { return lds_u32(SZX_TSCLAMP ? umin(ad, lastw) : ad); };
     const int lane = threadIdx.x & 31;
     const bool raw = RAWOK && R >= 32u;
     const uint32_t s = raw ? 0u : ((8u - (R & 7u)) & 7u);
@@ -1063,26 +1073,27 @@ __device__ __forceinline__ bool ts_decode_f32(uint32_t a, uint32_t R, uint32_t z
     const uint32_t mb = a + 33u, wp = mb & ~3u, pos0 = 8u * (mb & 3u);
     // window (lo, hi, nx) = words k, k+1, k+2 of the run from wp; pos = absolute
     // bit position from wp (lo holds bits [32 k, 32 k + 32)), lim = 32 (k + 1)
-    uint32_t lo = lds_u32(wp), hi = lds_u32(wp + 4), nx = lds_u32(wp + 8);
+    uint32_t lo = ldc(wp), hi = ldc(wp + 4), nx = ldc(wp + 8);
     uint32_t pos = pos0, lim = 32u, prev = 0;
     const uint32_t wp8 = wp + 8u;
     const uint32_t sw = ((uint32_t)lane >> 2) & 1u;     // transpose swizzle (bank-conflict free)
     // the lead codes: group g's 4 code bytes start at a + 1 + 4 g; the aligned
     // words cw0 (this group's first) and cw1 (next) are loaded a group ahead
     const uint32_t cb0 = (a + 1u) & ~3u, csh = 8u * (a + 1u);
-    uint32_t cw0 = lds_u32(cb0), cw1 = lds_u32(cb0 + 4u);
+    uint32_t cw0 = ldc(cb0), cw1 = ldc(cb0 + 4u);
 #pragma unroll 1
     for (int g = 0; g < 8; g++) {
         uint32_t cw = __funnelshift_r(cw0, cw1, csh);  // this group's 16 lead codes
         cw0 = cw1;
-        cw1 = lds_u32(cb0 + 8u + 4u * (uint32_t)g);    // (read past the codes on the last group: inside the payload / pad)
+        cw1 = ldc(cb0 + 8u + 4u * (uint32_t)g);        // (read past the codes on the last group: inside the payload / pad)
         cw ^= cw & (cw >> 1) & fix;
+        constexpr int FL = SZX_TSFL16 ? 16 : 8;   // values per transpose flush
 #pragma unroll
-        for (int h = 0; h < 2; h++) {
-            float o[8];
+        for (int h = 0; h < 16 / FL; h++) {
+            float o[FL];
 #pragma unroll
-            for (int i = 0; i < 8; i++) {
-                const int ii = 8 * h + i;
+            for (int i = 0; i < FL; i++) {
+                const int ii = FL * h + i;
                 // step 2: c8 = 8 x bytes copied from the previous value; step 3: m8 = 8 x mid-bytes
                 const uint32_t c8 = ii == 0 ? (cw << 3) & 24u : ii == 1 ? (cw << 1) & 24u : (cw >> (2 * ii - 3)) & 24u;
                 const uint32_t nm = 0xFFFFFFFFu >> c8;
@@ -1104,9 +1115,12 @@ __device__ __forceinline__ bool ts_decode_f32(uint32_t a, uint32_t R, uint32_t z
                     "@q mov.b32 %1, %2;\n\t"
                     "shr.u32 ad, %3, 3;\n\t"
                     "add.u32 ad, ad, %5;\n\t"
+#if SZX_TSCLAMP
+                    "min.u32 ad, ad, %6;\n\t"
+#endif
                     "@q ld.shared.u32 %2, [ad];\n\t}"
                     : "+r"(lo), "+r"(hi), "+r"(nx), "+r"(lim)
-                    : "r"(pos), "r"(wp8 - 4u)
+                    : "r"(pos), "r"(wp8 - 4u), "r"(lastw)
                     : "memory");
 #elif SZX_TSUNC
                 // slide one word (m8 <= 32: at most one per value); nx is re-read
@@ -1125,6 +1139,27 @@ __device__ __forceinline__ bool ts_decode_f32(uint32_t a, uint32_t R, uint32_t z
                 }
 #endif
             }
+#if SZX_TSFL16
+            // 32 blocks x 16 values through 2 KB: lane j's chunk c at row j, slot c ^ ((j >> 1) & 3);
+            // read back as 8 blocks x 64 bytes per store instruction
+            {
+                const uint32_t row = tb + 64u * (uint32_t)lane, sz = ((uint32_t)lane >> 1) & 3u;
+#pragma unroll
+                for (int c = 0; c < 4; c++)
+                    asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(row + 16u * ((uint32_t)c ^ sz)),
+                                 "r"(__float_as_uint(o[4 * c])), "r"(__float_as_uint(o[4 * c + 1])),
+                                 "r"(__float_as_uint(o[4 * c + 2])), "r"(__float_as_uint(o[4 * c + 3])) : "memory");
+                __syncwarp();
+#pragma unroll
+                for (int k = 0; k < 4; k++) {
+                    const uint32_t b = ((uint32_t)lane >> 2) + 8u * (uint32_t)k, c = (uint32_t)lane & 3u;
+                    const uint4 v = lds_u128(tb + 64u * b + 16u * (c ^ ((b >> 1) & 3u)));
+                    if ((word >> b) & 1u)
+                        st_out16(reinterpret_cast<uint4*>(yt + 128u * b + 16u * (uint32_t)g + 4u * c), v);
+                }
+                __syncwarp();
+            }
+#else
             const uint32_t row = tb + 32u * (uint32_t)lane;
             asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(row + 16u * sw), "r"(__float_as_uint(o[0])),
                          "r"(__float_as_uint(o[1])), "r"(__float_as_uint(o[2])), "r"(__float_as_uint(o[3])) : "memory");
@@ -1139,6 +1174,7 @@ __device__ __forceinline__ bool ts_decode_f32(uint32_t a, uint32_t R, uint32_t z
                     st_out16(reinterpret_cast<uint4*>(yt + 128u * b + 16u * (uint32_t)g + 8u * (uint32_t)h + 4u * c), v);
             }
             __syncwarp();
+#endif
         }
     }
     // the block's mid-bytes end exactly at its zsize
@@ -1652,8 +1688,9 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 8 && VPL == 4) ? SZX_DMINB6
                     float* yt = reinterpret_cast<float*>(y) + t * TB * B;
                     const float mu = __uint_as_float((uint32_t)cur.mul);
                     bool ok;
-                    if (__any_sync(0xffffffffu, R >= 32u)) ok = ts_decode_f32<true>(a, R, has ? zz : 33u, mu, tb, yt, cur.word);
-                    else ok = ts_decode_f32<false>(a, R, has ? zz : 33u, mu, tb, yt, cur.word);
+                    const uint32_t lastw = region + C::REGION - 4u;
+                    if (__any_sync(0xffffffffu, R >= 32u)) ok = ts_decode_f32<true>(a, R, has ? zz : 33u, mu, tb, yt, cur.word, lastw);
+                    else ok = ts_decode_f32<false>(a, R, has ? zz : 33u, mu, tb, yt, cur.word, lastw);
                     if (has && (bad || !ok)) set_corrupt(p.err);
                 } else if (t < nW_full) {
                     // segment decoder, one segment at a time
