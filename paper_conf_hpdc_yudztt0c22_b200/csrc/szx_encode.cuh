@@ -76,6 +76,12 @@ __device__ inline uint64_t gtimer() {
 #define SZX_ETL(tile, k) do { } while (0)
 #endif
 
+#ifndef SZX_EXP_NOCOPY
+#define SZX_EXP_NOCOPY 0  // timing experiments only (invalid streams): skip the copy-out
+#endif
+#ifndef SZX_EXP_NOPACK
+#define SZX_EXP_NOPACK 0  // timing experiments only (invalid streams): skip the pack
+#endif
 #ifndef SZX_GUARDSTAT
 #define SZX_GUARDSTAT 0  // diagnostic builds: count blocks whose R2 guard runs in the fused encoder
 #endif
@@ -464,7 +470,7 @@ __global__ void __launch_bounds__(32 * NW + 32, sizeof(T) == 4 ? SZX_EMINB : SZX
             s_excl[sl] = pv & ~(1ull << 63);
         }
         bar_compute(C::NTC);
-        copy_out_tile<C::NTC>(slot_addr(sl), out + off_pl + s_excl[sl], s_T[sl]);
+        if (!SZX_EXP_NOCOPY) copy_out_tile<C::NTC>(slot_addr(sl), out + off_pl + s_excl[sl], s_T[sl]);
         if (tid == 0) SZX_ETL(s_tile[sl], 3);
         // (the slot is zeroed when it is reused, NS - 1 tiles later)
     };
@@ -629,7 +635,7 @@ __global__ void __launch_bounds__(32 * NW + 32, sizeof(T) == 4 ? SZX_EMINB : SZX
             }
             zex = incl - zl;
             if (fast) {
-                if (valid) {
+                if (valid && !SZX_EXP_NOPACK) {
                     if constexpr (sizeof(T) == 4) quarter_pack_f32(e, m8, R, mexcl, stg + zoff);
                     else quarter_pack_f64(e, m8, R, mexcl, stg + zoff);
                 }
