@@ -21,6 +21,8 @@
 //         associative.
 #pragma once
 
+#include <utility>
+
 #include "szx_device.cuh"
 
 namespace szx {
@@ -1000,6 +1002,9 @@ struct DecWCfg {
 #ifndef SZX_TSFL16
 #define SZX_TSFL16 1   // thread-serial decoder: transpose 16 values per flush (64-byte block segments)
 #endif
+#ifndef SZX_TSFL
+#define SZX_TSFL 16    // values per transpose flush (32: 4 KB buffer, whole-line stores; needs a larger region)
+#endif
 #ifndef SZX_TSCLAMP
 #define SZX_TSCLAMP 1  // thread-serial decoder: payload reads clamped to the warp's region (no over-read pad)
 #endif
@@ -1018,7 +1023,7 @@ struct DecWCfg {
     // per-warp shared region: the two staging slots of the segment decoder, or
     // (thread-serial tiles) a 1 KB transpose buffer + one staging area + over-read pad
     static constexpr int REGION = SZX_DREGION > 2 * SLOT_ALLOC ? SZX_DREGION : 2 * SLOT_ALLOC;
-    static constexpr int TS_TB = SZX_TSFL16 ? 2048 : 1024;  // transpose buffer: 32 blocks x 16 (8) values
+    static constexpr int TS_TB = SZX_TSFL == 32 ? 4096 : SZX_TSFL16 ? 2048 : 1024;  // transpose buffer: 32 blocks x FL values
     static constexpr int TS_PAD = SZX_TSCLAMP ? 16 : 576;   // reads clamped to the region, or > 12 + 128 x 4
                                                             // bytes a corrupt lane may over-read
     static constexpr int TS_STAGE = REGION - TS_TB - TS_PAD;
@@ -1057,6 +1062,11 @@ __device__ uint64_t g_tl[kTlCtas * 8 * 4];
 // tb: 1 KB transpose buffer; yt: the tile's first output value; word: the
 // tile's nonconstant bitmap (lanes of constant blocks run on dummy input and
 // store nothing).  Returns false (this lane) on a size mismatch.
+template <int... Is, typename F>
+__device__ __forceinline__ void unroll_i_impl(F&& f, std::integer_sequence<int, Is...>) { (f(std::integral_constant<int, Is>{}), ...); }
+template <int N, typename F>
+__device__ __forceinline__ void unroll_i(F&& f) { unroll_i_impl(f, std::make_integer_sequence<int, N>{}); }
+
 template <bool RAWOK>
 __device__ __forceinline__ bool ts_decode_f32(uint32_t a, uint32_t R, uint32_t zz, float mu, uint32_t tb,
                                               float* __restrict__ yt, uint32_t word, uint32_t lastw) {
@@ -1081,64 +1091,103 @@ __device__ __forceinline__ bool ts_decode_f32(uint32_t a, uint32_t R, uint32_t z
     // words cw0 (this group's first) and cw1 (next) are loaded a group ahead
     const uint32_t cb0 = (a + 1u) & ~3u, csh = 8u * (a + 1u);
     uint32_t cw0 = ldc(cb0), cw1 = ldc(cb0 + 4u);
+    // one value (index II of its 16-value code group, codes cw): Fig. 10 steps 2-5
+    auto value = [&](auto IIc, uint32_t cw) -> float {
+        constexpr int II = decltype(IIc)::value;
+            // step 2: c8 = 8 x bytes copied from the previous value; step 3: m8 = 8 x mid-bytes
+            const uint32_t c8 = II == 0 ? (cw << 3) & 24u : II == 1 ? (cw << 1) & 24u : (cw >> (2 * II - 3)) & 24u;
+            const uint32_t nm = 0xFFFFFFFFu >> c8;
+            const uint32_t m8 = r8 - c8;
+            const uint32_t mid = __funnelshift_r(lo, hi, pos);
+            const uint32_t w = bitsel(prev, mid * pdrop, nm);  // steps 2-4
+            prev = w;
+            const float ov = raw ? __uint_as_float(w) : __fadd_rn(__uint_as_float(w * ps), mu);  // step 5
+            pos += m8;
+#if SZX_TSASM
+            // slide one word (m8 <= 32: at most one per value), in one PTX
+            // block so the predicated load lands in nx itself (no move of a
+            // just-loaded register)
+            asm volatile(
+                "{\n\t.reg .pred q;\n\t.reg .u32 ad;\n\t"
+                "setp.ge.u32 q, %4, %3;\n\t"
+                "@q add.u32 %3, %3, 32;\n\t"
+                "@q mov.b32 %0, %1;\n\t"
+                "@q mov.b32 %1, %2;\n\t"
+                "shr.u32 ad, %3, 3;\n\t"
+                "add.u32 ad, ad, %5;\n\t"
+#if SZX_TSCLAMP
+                "min.u32 ad, ad, %6;\n\t"
+#endif
+                "@q ld.shared.u32 %2, [ad];\n\t}"
+                : "+r"(lo), "+r"(hi), "+r"(nx), "+r"(lim)
+                : "r"(pos), "r"(wp8 - 4u), "r"(lastw)
+                : "memory");
+#elif SZX_TSUNC
+            // slide one word (m8 <= 32: at most one per value); nx is re-read
+            // every value (unpredicated: no move of a just-loaded register)
+            const bool sl = pos >= lim;
+            lim += sl ? 32u : 0u;
+            lo = sl ? hi : lo;
+            hi = sl ? nx : hi;
+            nx = lds_u32(wp8 + (lim >> 3) - 4u);
+#else
+            if (pos >= lim) {  // slide one word (m8 <= 32: at most one per value)
+                lim += 32u;
+                lo = hi;
+                hi = nx;
+                nx = lds_u32(wp8 + (lim >> 3) - 4u);  // word k + 2 of the new window
+            }
+#endif
+        return ov;
+    };
+#if SZX_TSFL == 32
+    // 32 values per flush: two code groups, then 32 blocks x 32 values through 4 KB
+    // (lane j's chunk c at row j, slot c ^ (j & 7)), stored as 4 blocks x 128 bytes
+    // (whole lines) per store instruction
+#pragma unroll 1
+    for (int f = 0; f < 4; f++) {
+        float o[32];
+        unroll_i<2>([&](auto Gc) {
+            constexpr int gg = decltype(Gc)::value;
+            uint32_t cw = __funnelshift_r(cw0, cw1, csh);
+            cw0 = cw1;
+            cw1 = ldc(cb0 + 8u + 4u * (uint32_t)(2 * f + gg));
+            cw ^= cw & (cw >> 1) & fix;
+            unroll_i<16>([&](auto I) {
+                constexpr int i = decltype(I)::value;
+                o[16 * gg + i] = value(std::integral_constant<int, i>{}, cw);
+            });
+        });
+        const uint32_t row = tb + 128u * (uint32_t)lane, sz = (uint32_t)lane & 7u;
+#pragma unroll
+        for (int c = 0; c < 8; c++)
+            asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(row + 16u * ((uint32_t)c ^ sz)),
+                         "r"(__float_as_uint(o[4 * c])), "r"(__float_as_uint(o[4 * c + 1])),
+                         "r"(__float_as_uint(o[4 * c + 2])), "r"(__float_as_uint(o[4 * c + 3])) : "memory");
+        __syncwarp();
+#pragma unroll
+        for (int k = 0; k < 8; k++) {
+            const uint32_t b = ((uint32_t)lane >> 3) + 4u * (uint32_t)k, c = (uint32_t)lane & 7u;
+            const uint4 v = lds_u128(tb + 128u * b + 16u * (c ^ (b & 7u)));
+            if ((word >> b) & 1u) st_out16(reinterpret_cast<uint4*>(yt + 128u * b + 32u * (uint32_t)f + 4u * c), v);
+        }
+        __syncwarp();
+    }
+#else
 #pragma unroll 1
     for (int g = 0; g < 8; g++) {
         uint32_t cw = __funnelshift_r(cw0, cw1, csh);  // this group's 16 lead codes
         cw0 = cw1;
         cw1 = ldc(cb0 + 8u + 4u * (uint32_t)g);        // (read past the codes on the last group: inside the payload / pad)
         cw ^= cw & (cw >> 1) & fix;
-        constexpr int FL = SZX_TSFL16 ? 16 : 8;   // values per transpose flush
-#pragma unroll
-        for (int h = 0; h < 16 / FL; h++) {
+        constexpr int FL = SZX_TSFL16 ? 16 : 8;   // values per transpose flush (SZX_TSFL == 32: below)
+        unroll_i<16 / FL>([&](auto Hc) {
+            constexpr int h = decltype(Hc)::value;
             float o[FL];
-#pragma unroll
-            for (int i = 0; i < FL; i++) {
-                const int ii = FL * h + i;
-                // step 2: c8 = 8 x bytes copied from the previous value; step 3: m8 = 8 x mid-bytes
-                const uint32_t c8 = ii == 0 ? (cw << 3) & 24u : ii == 1 ? (cw << 1) & 24u : (cw >> (2 * ii - 3)) & 24u;
-                const uint32_t nm = 0xFFFFFFFFu >> c8;
-                const uint32_t m8 = r8 - c8;
-                const uint32_t mid = __funnelshift_r(lo, hi, pos);
-                const uint32_t w = bitsel(prev, mid * pdrop, nm);  // steps 2-4
-                prev = w;
-                o[i] = raw ? __uint_as_float(w) : __fadd_rn(__uint_as_float(w * ps), mu);  // step 5
-                pos += m8;
-#if SZX_TSASM
-                // slide one word (m8 <= 32: at most one per value), in one PTX
-                // block so the predicated load lands in nx itself (no move of a
-                // just-loaded register)
-                asm volatile(
-                    "{\n\t.reg .pred q;\n\t.reg .u32 ad;\n\t"
-                    "setp.ge.u32 q, %4, %3;\n\t"
-                    "@q add.u32 %3, %3, 32;\n\t"
-                    "@q mov.b32 %0, %1;\n\t"
-                    "@q mov.b32 %1, %2;\n\t"
-                    "shr.u32 ad, %3, 3;\n\t"
-                    "add.u32 ad, ad, %5;\n\t"
-#if SZX_TSCLAMP
-                    "min.u32 ad, ad, %6;\n\t"
-#endif
-                    "@q ld.shared.u32 %2, [ad];\n\t}"
-                    : "+r"(lo), "+r"(hi), "+r"(nx), "+r"(lim)
-                    : "r"(pos), "r"(wp8 - 4u), "r"(lastw)
-                    : "memory");
-#elif SZX_TSUNC
-                // slide one word (m8 <= 32: at most one per value); nx is re-read
-                // every value (unpredicated: no move of a just-loaded register)
-                const bool sl = pos >= lim;
-                lim += sl ? 32u : 0u;
-                lo = sl ? hi : lo;
-                hi = sl ? nx : hi;
-                nx = lds_u32(wp8 + (lim >> 3) - 4u);
-#else
-                if (pos >= lim) {  // slide one word (m8 <= 32: at most one per value)
-                    lim += 32u;
-                    lo = hi;
-                    hi = nx;
-                    nx = lds_u32(wp8 + (lim >> 3) - 4u);  // word k + 2 of the new window
-                }
-#endif
-            }
+            unroll_i<FL>([&](auto I) {
+                constexpr int i = decltype(I)::value;
+                o[i] = value(std::integral_constant<int, FL * h + i>{}, cw);
+            });
 #if SZX_TSFL16
             // 32 blocks x 16 values through 2 KB: lane j's chunk c at row j, slot c ^ ((j >> 1) & 3);
             // read back as 8 blocks x 64 bytes per store instruction
@@ -1175,8 +1224,9 @@ __device__ __forceinline__ bool ts_decode_f32(uint32_t a, uint32_t R, uint32_t z
             }
             __syncwarp();
 #endif
-        }
+        });
     }
+#endif
     // the block's mid-bytes end exactly at its zsize
     return pos - pos0 == 8u * (zz - 33u);
 }
