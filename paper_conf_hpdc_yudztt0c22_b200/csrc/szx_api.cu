@@ -382,6 +382,9 @@ void enqueue_encode(const void* d_in, const Plan& p, const CLayout& L, uint8_t* 
 #ifndef SZX_DITEMS
 #define SZX_DITEMS 2        // decoder: target nonconstant work items per decode warp (tile split)
 #endif
+#ifndef SZX_DTS_MINT
+#define SZX_DTS_MINT 4      // ... only with at least this many tiles per warp of the grid
+#endif
 #ifndef SZX_DTS
 #define SZX_DTS 1           // decoder: thread-serial tiles on dense float32 b = 128 streams
 #endif
@@ -583,8 +586,12 @@ int enqueue_decompress(const void* d_in, uint64_t in_bytes, const szx_header_t* 
             if (SZX_DSPLIT) p.split = SZX_DSPLIT;
             // dense float32 b = 128 streams: the thread-serial tile decoder (a
             // performance choice only; the device validates the stream itself)
+            // (at least SZX_DTS_MINT tiles per warp of the grid: a lane-per-block tile takes
+            // a warp as long as a whole tile, so few tiles per warp leave a long tail --
+            // Hurricane's 6,103 tiles decode faster with the half-warp form)
             p.ts = (SZX_DTS && sizeof(T) == 4 && V == 4 && !d_ref && p.split == 1 && kb0 == 0 &&
-                    kb1 == L.nB && 4 * h->n_nonconst >= 3 * L.nB) ? 1u : 0u;
+                    kb1 == L.nB && 4 * h->n_nonconst >= 3 * L.nB &&
+                    p.nWi >= (uint64_t)SZX_DTS_MINT * gcap * DecWCfg<T, V>::NWARP) ? 1u : 0u;
             uint64_t grid = cdiv(p.nWi * p.split, 8);
             if (grid > gcap) grid = gcap;
             // index CTAs: at most one per SM, and at most one 256-tile chunk each

@@ -49,10 +49,10 @@ x = synth.nyx_like(0, n=32).reshape(-1).cuda()
 mm = szx.local_minmax(x)
 e = (1e-3 * (mm[1] - mm[0])).reshape(1).contiguous()
 s = szx.compress_shard(x, 1e-3, e, "rel", 128)
-# the dense float32 decoder loop (thread-serial tiles; >= ~22 M values): mixed tile shapes,
+# the dense float32 decoder loop (thread-serial tiles; >= ~58 M values): mixed tile shapes,
 # a raw block and an all-constant tile, decoded once (SANITIZE_TS=0 skips it)
 if os.environ.get("SANITIZE_TS", "1") == "1":
-    xt = synth.nyx_like(1, n=288).reshape(-1).numpy().copy()[:-77]
+    xt = synth.nyx_like(1, n=400).reshape(-1).numpy().copy()[:-77]
     nW = xt.size // 4096
     blk = xt[: nW * 4096].reshape(nW, 32, 128)
     blk[3::7, :6, :] = 1.5e6
