@@ -18,6 +18,8 @@ elif cfg == "qmcpack":
     x, eb = synth.qmcpack_like(device="cuda").reshape(-1).contiguous(), 1e-4
 elif cfg == "cesm":
     x = synth.cesm_like(field, device="cuda").reshape(-1).contiguous()
+elif cfg == "hacc":
+    x = synth.hacc_like(field, device="cuda").reshape(-1).contiguous()
 elif cfg == "hurricane":
     x = synth.hurricane_like(field, device="cuda").reshape(-1).contiguous()
 else:
